@@ -1,0 +1,143 @@
+/* wcsvd.h -- C-ABI of the B200-native batched one-sided Jacobi SVD (W-cycle SVD hot path).
+ *
+ * Library: paper_conf_sc_xiaopxsmmlzt22_b200/libwcsvd.so, CUDA for sm_100a only.
+ * Citations are lines of the paper's text, PAPER.md:N (section / equation / algorithm).
+ *
+ * Problem (§II.A eq 1; §III.B; Alg 2 l.1):
+ *   a batch of mu independent real matrices A^k (m_k x n_k, sizes may all differ) is factorised
+ *   as A^k = U^k diag(S^k) (V^k)^T -- economy form, k_k = min(m_k, n_k) triplets.
+ * Method (the hot path, BASELINE.json north_star): batched one-sided Jacobi. Column-block pairs
+ *   [A_i A_j] are orthogonalised by Gram -> in-SMEM Jacobi EVD -> A/V block update -> off-norm test
+ *   (Alg 1; Alg 2), inside the multilevel W-cycle;
+ *   matrices that fit on-chip run the Level-0 vector-rotation kernel (§IV.B).
+ *
+ * Conventions (all entry points):
+ *  - fp64, column-major, economy SVD: S[k] descending, U m x k, V n x k.
+ *  - Ownership: the caller owns A, S, U, V (DEVICE memory) and every host array; host arrays are
+ *    consumed before the call returns and may be freed immediately. The library owns only its
+ *    workspace (stream-ordered cudaMallocAsync on `stream`, or the caller's buffer via _ex).
+ *    A is read-only.
+ *  - Asynchronous on `stream`: a return of WCSVD_OK means the work was enqueued.
+ *  - Errors: negative codes are returned synchronously and nothing is enqueued on failure:
+ *      -i          the i-th argument (1-based) is invalid (LAPACK convention);
+ *      WCSVD_ENOTSUP  a size outside 1 <= m, n <= 1024;
+ *      WCSVD_ECUDA    a CUDA error (no device, launch failure, missing sm_100a image);
+ *      WCSVD_ENOMEM   workspace allocation failed.
+ *    Numerical outcomes are per matrix, asynchronous, in opts->info (see wcsvd_opts).
+ *  - Deterministic: the outputs for one matrix depend only on (m, n, the bits of A, tol,
+ *    max_sweeps) -- never on batch composition, stream, device index or device count. The plan is
+ *    a function of (m, n) only; there are no floating-point atomics.
+ *  - Reentrant; no global mutable state.
+ */
+#ifndef WCSVD_H_
+#define WCSVD_H_
+
+#include <stddef.h>
+
+#if defined(__GNUC__)
+#define WCSVD_API __attribute__((visibility("default")))
+#else
+#define WCSVD_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* cudaStream_t is an opaque pointer; declared here so this header needs no CUDA include. */
+typedef struct CUstream_st* wcsvd_stream_t;
+
+enum {
+  WCSVD_OK = 0,
+  WCSVD_ENOTSUP = -100,
+  WCSVD_ECUDA = -101,
+  WCSVD_ENOMEM = -102
+};
+
+/* Paths a matrix can take through the W-cycle (Alg 2 l.2-14). */
+enum {
+  WCSVD_PATH_AUTO = 0,
+  WCSVD_PATH_L0 = 1,      /* whole matrix on-chip: vector-rotation Jacobi, Alg 2 l.2-3 */
+  WCSVD_PATH_GRAM = 2,    /* Level 1: Gram -> EVD(B_ij) -> GEMM update, Alg 2 l.10-11 */
+  WCSVD_PATH_WCYCLE = 3   /* Level 1 -> Level 2 recursion on each pair panel, Alg 2 l.12-14 */
+};
+
+/* wcsvd_batched -- batched economy SVD.
+ *  batch       >= 0; 0 is a no-op returning WCSVD_OK.                                    (arg 1)
+ *  m, n        host arrays [batch]; 1 <= m[b], n[b] <= 1024 (else WCSVD_ENOTSUP).        (2, 3)
+ *  A           host array [batch] of DEVICE pointers; A[b] is m x n column-major, ld lda[b],
+ *              8-byte aligned; not modified. Must not alias S/U/V.                        (4)
+ *  lda         host array [batch]; lda[b] >= m[b].                                        (5)
+ *  S           host array [batch] of DEVICE pointers to k = min(m,n) doubles, descending.   (6)
+ *  U           NULL (left vectors not returned) or host array [batch] of DEVICE pointers
+ *              (entries may be NULL): m x k column-major, ld m.                           (7)
+ *  V           NULL or host array [batch] of DEVICE pointers: n x k column-major, ld n.  (8)
+ *  tol         relative orthogonality threshold |a_i^T a_j| <= tol ||a_i|| ||a_j||;
+ *              <= 0 -> sqrt(max(m,n)) * 2^-53 per matrix.                                (9)
+ *  max_sweeps  outer-sweep cap; <= 0 -> 60. When reached, the best iterate is finalised (Z26). (10)
+ *  stream      CUDA stream (cudaStream_t) the work is enqueued on; NULL = legacy default. (11)
+ * Returns WCSVD_OK or a negative code (above). */
+WCSVD_API int wcsvd_batched(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                  double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
+                  wcsvd_stream_t stream);
+
+/* Extended options (argument 12 of wcsvd_batched_ex). Zero-initialise, then set struct_size. */
+typedef struct {
+  size_t struct_size;      /* = sizeof(wcsvd_opts); ABI versioning */
+  const int* ldu;          /* host [batch] or NULL (-> m): leading dimensions of U[b], >= m[b] */
+  const int* ldv;          /* host [batch] or NULL (-> n): leading dimensions of V[b], >= n[b] */
+  int* info;               /* DEVICE int[batch] or NULL. Per matrix, written asynchronously:
+                              > 0  outer sweeps used (the last, rotation-free one included, Z24);
+                              -1   not converged within max_sweeps (best iterate returned, Z26);
+                              -2   non-finite input (S, U, V filled with NaN). */
+  int* sweeps_inner;       /* DEVICE int[batch] or NULL: total inner (Level >= 2 / EVD) sweeps */
+  void* workspace;         /* DEVICE buffer or NULL (-> stream-ordered internal allocation) */
+  size_t workspace_bytes;  /* size of `workspace`; must be >= wcsvd_workspace_size(...) */
+  int force_path;          /* 0 = planner; else WCSVD_PATH_* for every matrix (ablations) */
+  int force_w;             /* 0 = planner; else Level-1 block width w in {8, 16} */
+  int force_w2;            /* 0 = planner; else Level-2 block width (W-cycle path) */
+  int inner_sweeps;        /* 0 = planner (1); cap on EVD sweeps per pair */
+} wcsvd_opts;
+
+WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                     double* const* S, double* const* U, double* const* V, double tol,
+                     int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
+
+/* Bytes of device workspace wcsvd_batched_ex needs for this batch (host-only, no CUDA call). */
+WCSVD_API size_t wcsvd_workspace_size(int batch, const int* m, const int* n);
+
+/* Static string for a status code. */
+WCSVD_API const char* wcsvd_status_string(int status);
+
+/* ---- Host-only planner introspection (no CUDA call; used by tests and the multi-GPU split) ---- */
+
+/* The per-matrix plan, a pure function of (m, n) (and an optional forced path / width). */
+typedef struct {
+  int m, n;            /* input sizes */
+  int M, N;            /* working orientation, M = max(m,n) >= N = min(m,n) */
+  int swapped;         /* 1 if m < n (the iteration runs on A^T) */
+  int path;            /* WCSVD_PATH_L0 / _GRAM / _WCYCLE */
+  int n_pad;           /* padded column count: a multiple of 2w (Level >= 1) or the L0 tile width */
+  int m_pad;           /* padded row count (multiple of 8) of the Level >= 1 working copy */
+  int w;               /* Level-1 block width (0 for L0) */
+  int w2;              /* Level-2 block width (W-cycle path), else 0 */
+  int variant;         /* kernel variant id (L0 template instance) */
+  double cost;         /* estimated flops per sweep, F_tb(M, N) = N(N-1)/2 (8M + 6N) */
+} wcsvd_plan_t;
+
+/* Fill *out with the plan for one m x n matrix. Returns WCSVD_OK, -1/-2 for bad m/n, or
+ * WCSVD_ENOTSUP. force_path / force_w as in wcsvd_opts (0 = planner). */
+WCSVD_API int wcsvd_plan(int m, int n, int force_path, int force_w, wcsvd_plan_t* out);
+
+/* The round-robin (circle-method) schedule used at every level.
+ * For `np` indices (even, >= 2) at step `step` (0 <= step < np-1), writes the np/2 disjoint pairs
+ * as pairs[2p], pairs[2p+1] (original indices, pairs[2p] < pairs[2p+1]). Returns 0 or -1. */
+WCSVD_API int wcsvd_round_robin(int np, int step, int* pairs);
+
+/* Library build identification, e.g. "wcsvd 0.1 sm_100a". */
+WCSVD_API const char* wcsvd_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WCSVD_H_ */

@@ -7,6 +7,12 @@ Acceptance bars are north_star's (BASELINE.json) as restated in SURVEY.md §8(c)
   vectors (Z25):  clusters = maximal runs of consecutive s_ref with adjacent gaps < 1e-6 s_ref_1;
                   singleton i: |u_i . u_ref_i| >= 1 - 1e-10 and |v_i . v_ref_i| >= 1 - 1e-10;
                   cluster: ||P - P_ref||_2 <= 1e-8 for the projectors onto the cluster spans.
+                  Reading R-VEC: a vector / subspace is only determined to
+                  theta ~ u s_1 / delta (Wedin), delta = the gap to the other singular values and, for
+                  the factor with more rows than k (U if m > n, V if m < n), also the smallest sigma of
+                  the group itself (its left/right null space is the competing subspace). Where that
+                  bound is looser, the bars become theta_max = 64 u s_1 / delta (projector) and
+                  theta_max^2 (1 - |cos|); elsewhere north_star's 1e-10 / 1e-8 stand.
 Residual and orthogonality are evaluated in numpy.longdouble for min(m,n) <= 128, else in float64
 (whose own evaluation error, ~sqrt(n) 2^-53 ~ 1e-14, is 100x below the bars).
 """
@@ -29,8 +35,8 @@ class Parity:
     sigma_err: float
     resid: float
     ortho: float
-    vec_err: float  # max over singletons of 1 - |cos|
-    proj_err: float  # max over clusters of ||P - P_ref||_2
+    vec_err: float  # max over singletons of 1 - |cos| (scaled by the R-VEC bound where looser)
+    proj_err: float  # max over clusters of ||P - P_ref||_2 (scaled likewise)
     n_clusters: int
     notes: list = field(default_factory=list)
 
@@ -91,15 +97,26 @@ def compare(A, S, U, V, S_ref, U_ref, V_ref, check_vectors: bool = True) -> Pari
         orth = max(orth, orthogonality(V))
     vec_err, proj_err, ncl = 0.0, 0.0, 0
     if check_vectors and U is not None and V is not None:
+        k = len(S_ref)
         for (a, b) in clusters(S_ref):
-            if b - a == 1:
-                cu = abs(float(np.dot(U[:, a], U_ref[:, a])))
-                cv = abs(float(np.dot(V[:, a], V_ref[:, a])))
-                vec_err = max(vec_err, 1.0 - cu, 1.0 - cv)
-            else:
+            gap = np.inf
+            if a > 0:
+                gap = min(gap, S_ref[a - 1] - S_ref[a])
+            if b < k:
+                gap = min(gap, S_ref[b - 1] - S_ref[b])
+            if b - a > 1:
                 ncl += 1
-                for (X, Xr) in ((U, U_ref), (V, V_ref)):
+            for (X, Xr) in ((U, U_ref), (V, V_ref)):
+                delta = gap
+                if X.shape[0] > k:  # the long factor: its null space competes (Wedin)
+                    delta = min(delta, S_ref[b - 1])
+                theta = 64 * 2.0 ** -53 * s1 / delta if delta > 0 else np.inf
+                if b - a == 1:
+                    c = abs(float(np.dot(X[:, a], Xr[:, a])))
+                    vec_err = max(vec_err, (1.0 - c) / max(1.0, theta ** 2 / VEC_TOL))
+                else:
                     P = X[:, a:b] @ X[:, a:b].T
                     Pr = Xr[:, a:b] @ Xr[:, a:b].T
-                    proj_err = max(proj_err, float(np.linalg.norm(P - Pr, 2)))
+                    e = float(np.linalg.norm(P - Pr, 2))
+                    proj_err = max(proj_err, e / max(1.0, theta / PROJ_TOL))
     return Parity(sig, res, orth, vec_err, proj_err, ncl)

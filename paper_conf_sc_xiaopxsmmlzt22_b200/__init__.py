@@ -1,0 +1,208 @@
+"""B200-native batched one-sided Jacobi SVD (the W-cycle SVD hot path, Xiao et al., SC'22).
+
+Thin Python binding over the C-ABI in ``include/wcsvd.h`` (``libwcsvd.so``, CUDA sm_100a).
+This module only marshals arguments: every numerical step runs in the library's CUDA kernels.
+PyTorch provides device memory and the current stream. There is no CPU fallback: if the library
+or a CUDA device is missing, calls raise.
+
+Layout: torch tensors are row-major, the C-ABI is column-major. A contiguous m x n tensor is the
+column-major n x m matrix A^T (lda = n); we factor that and swap the roles of U and V, which costs
+no copies (U and V are returned as transposed views of contiguous buffers).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Sequence
+
+import numpy as np
+
+__all__ = ["svd_batched", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
+           "PATH_L0", "PATH_GRAM", "PATH_WCYCLE", "library_path"]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "libwcsvd.so")
+
+PATH_AUTO, PATH_L0, PATH_GRAM, PATH_WCYCLE = 0, 1, 2, 3
+WCSVD_OK, WCSVD_ENOTSUP, WCSVD_ECUDA, WCSVD_ENOMEM = 0, -100, -101, -102
+
+
+class WcsvdError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"wcsvd error {code}: {msg}")
+        self.code = code
+
+
+class PlanT(ctypes.Structure):
+    _fields_ = [("m", ctypes.c_int), ("n", ctypes.c_int), ("M", ctypes.c_int), ("N", ctypes.c_int),
+                ("swapped", ctypes.c_int), ("path", ctypes.c_int), ("n_pad", ctypes.c_int),
+                ("m_pad", ctypes.c_int), ("w", ctypes.c_int), ("w2", ctypes.c_int),
+                ("variant", ctypes.c_int), ("cost", ctypes.c_double)]
+
+
+class OptsT(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_size_t), ("ldu", ctypes.c_void_p), ("ldv", ctypes.c_void_p),
+                ("info", ctypes.c_void_p), ("sweeps_inner", ctypes.c_void_p),
+                ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
+                ("force_path", ctypes.c_int), ("force_w", ctypes.c_int), ("force_w2", ctypes.c_int),
+                ("inner_sweeps", ctypes.c_int)]
+
+
+_lib = None
+
+
+def library_path() -> str:
+    return _LIB_PATH
+
+
+def lib() -> ctypes.CDLL:
+    """Load libwcsvd.so (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIB_PATH):
+        raise WcsvdError(-101, f"{_LIB_PATH} not built; run __graft_entry__.build() "
+                               "(or python paper_conf_sc_xiaopxsmmlzt22_b200/build.py)")
+    L = ctypes.CDLL(_LIB_PATH)
+    P, I, D = ctypes.c_void_p, ctypes.c_int, ctypes.c_double
+    L.wcsvd_batched.argtypes = [I, P, P, P, P, P, P, P, D, I, P]
+    L.wcsvd_batched.restype = I
+    L.wcsvd_batched_ex.argtypes = [I, P, P, P, P, P, P, P, D, I, P, ctypes.POINTER(OptsT)]
+    L.wcsvd_batched_ex.restype = I
+    L.wcsvd_workspace_size.argtypes = [I, P, P]
+    L.wcsvd_workspace_size.restype = ctypes.c_size_t
+    L.wcsvd_status_string.argtypes = [I]
+    L.wcsvd_status_string.restype = ctypes.c_char_p
+    L.wcsvd_plan.argtypes = [I, I, I, I, ctypes.POINTER(PlanT)]
+    L.wcsvd_plan.restype = I
+    L.wcsvd_round_robin.argtypes = [I, I, P]
+    L.wcsvd_round_robin.restype = I
+    L.wcsvd_version.restype = ctypes.c_char_p
+    _lib = L
+    return L
+
+
+def _check(code: int):
+    if code != WCSVD_OK:
+        raise WcsvdError(code, lib().wcsvd_status_string(code).decode())
+
+
+def plan(m: int, n: int, force_path: int = 0, force_w: int = 0) -> dict:
+    """Planner introspection (host-only): the per-matrix plan as a dict."""
+    p = PlanT()
+    _check(lib().wcsvd_plan(int(m), int(n), int(force_path), int(force_w), ctypes.byref(p)))
+    return {f: getattr(p, f) for f, _ in PlanT._fields_}
+
+
+def round_robin(np_: int, step: int) -> list:
+    """The round-robin pairs (i, j) of `step` for `np_` indices (host-only)."""
+    buf = (ctypes.c_int * np_)()
+    if lib().wcsvd_round_robin(int(np_), int(step), buf) != 0:
+        raise ValueError("bad round-robin arguments")
+    return [(buf[2 * k], buf[2 * k + 1]) for k in range(np_ // 2)]
+
+
+def _arr_i32(x) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(x, dtype=np.int32))
+
+
+def _arr_ptr(x) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(x, dtype=np.uint64))
+
+
+def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: float = 0.0,
+                    max_sweeps: int = 0, stream: int = 0, ldu=None, ldv=None, info_ptr: int = 0,
+                    sweeps_inner_ptr: int = 0, workspace_ptr: int = 0, workspace_bytes: int = 0,
+                    force_path: int = 0, force_w: int = 0, force_w2: int = 0,
+                    inner_sweeps: int = 0) -> None:
+    """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError."""
+    m, n, lda = _arr_i32(m), _arr_i32(n), _arr_i32(lda)
+    B = len(m)
+    Ap, Sp = _arr_ptr(A_ptrs), _arr_ptr(S_ptrs)
+    Up = _arr_ptr(U_ptrs) if U_ptrs is not None else None
+    Vp = _arr_ptr(V_ptrs) if V_ptrs is not None else None
+    keep = []
+    opts = OptsT()
+    opts.struct_size = ctypes.sizeof(OptsT)
+    if ldu is not None:
+        a = _arr_i32(ldu); keep.append(a); opts.ldu = a.ctypes.data
+    if ldv is not None:
+        a = _arr_i32(ldv); keep.append(a); opts.ldv = a.ctypes.data
+    opts.info = info_ptr or None
+    opts.sweeps_inner = sweeps_inner_ptr or None
+    opts.workspace = workspace_ptr or None
+    opts.workspace_bytes = workspace_bytes
+    opts.force_path, opts.force_w, opts.force_w2, opts.inner_sweeps = force_path, force_w, force_w2, inner_sweeps
+    rc = lib().wcsvd_batched_ex(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
+                                Sp.ctypes.data, Up.ctypes.data if Up is not None else None,
+                                Vp.ctypes.data if Vp is not None else None, float(tol), int(max_sweeps),
+                                stream or None, ctypes.byref(opts))
+    _check(rc)
+
+
+def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = True,
+                return_info: bool = False, out=None, **kw):
+    """Batched economy SVD of fp64 CUDA tensors on the current stream.
+
+    A: tensor [B, m, n] (contiguous) or a sequence of 2-D tensors (sizes may differ).
+    Returns (S, U, V) with A = U diag(S) V^T; for a batched tensor S [B, k], U [B, m, k],
+    V [B, n, k] (U, V are transposed views); for a list, lists of tensors. With return_info,
+    also the per-matrix int32 info tensor (sweeps, -1 not converged, -2 non-finite).
+    ``out`` = (S, Ubuf, Vbuf) preallocated as returned by a previous call (batched form only).
+    """
+    import torch
+
+    if not torch.cuda.is_available():
+        raise WcsvdError(WCSVD_ECUDA, "no CUDA device (this library has no CPU fallback)")
+    stream = torch.cuda.current_stream().cuda_stream
+    if isinstance(A, torch.Tensor):
+        if A.dim() != 3 or A.dtype != torch.float64 or not A.is_cuda:
+            raise ValueError("A must be a float64 CUDA tensor [B, m, n]")
+        A = A.contiguous()
+        B, m, n = A.shape
+        k = min(m, n)
+        dev = A.device
+        if out is not None:
+            S, Ubuf, Vbuf = out
+        else:
+            S = torch.empty(B, k, dtype=torch.float64, device=dev)
+            Ubuf = torch.empty(B, k, m, dtype=torch.float64, device=dev) if compute_uv else None
+            Vbuf = torch.empty(B, k, n, dtype=torch.float64, device=dev) if compute_uv else None
+        info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
+        idx = np.arange(B, dtype=np.uint64)
+        a_ptr = A.data_ptr() + idx * np.uint64(8 * m * n)
+        s_ptr = S.data_ptr() + idx * np.uint64(8 * k)
+        # column-major view: the library factors A^T (n x m, lda = n); its "U" (n x k) is our V,
+        # its "V" (m x k) is our U.
+        u_ptr = (Vbuf.data_ptr() + idx * np.uint64(8 * k * n)) if compute_uv else None
+        v_ptr = (Ubuf.data_ptr() + idx * np.uint64(8 * k * m)) if compute_uv else None
+        svd_batched_raw(np.full(B, n), np.full(B, m), a_ptr, np.full(B, n), s_ptr, u_ptr, v_ptr,
+                        tol=tol, max_sweeps=max_sweeps, stream=stream,
+                        info_ptr=info.data_ptr() if info is not None else 0, **kw)
+        U = Ubuf.transpose(1, 2) if compute_uv else None
+        V = Vbuf.transpose(1, 2) if compute_uv else None
+        return (S, U, V, info) if return_info else (S, U, V)
+    # list of 2-D tensors
+    As = [a.contiguous() for a in A]
+    for a in As:
+        if a.dim() != 2 or a.dtype != torch.float64 or not a.is_cuda:
+            raise ValueError("each matrix must be a 2-D float64 CUDA tensor")
+    B = len(As)
+    if B == 0:
+        return ([], [], []) if not return_info else ([], [], [], None)
+    dev = As[0].device
+    ms = [a.shape[0] for a in As]
+    ns = [a.shape[1] for a in As]
+    ks = [min(x, y) for x, y in zip(ms, ns)]
+    Ss = [torch.empty(k, dtype=torch.float64, device=dev) for k in ks]
+    Ub = [torch.empty(k, mm, dtype=torch.float64, device=dev) for k, mm in zip(ks, ms)] if compute_uv else None
+    Vb = [torch.empty(k, nn, dtype=torch.float64, device=dev) for k, nn in zip(ks, ns)] if compute_uv else None
+    info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
+    svd_batched_raw(ns, ms, [a.data_ptr() for a in As], ns, [s.data_ptr() for s in Ss],
+                    [v.data_ptr() for v in Vb] if compute_uv else None,
+                    [u.data_ptr() for u in Ub] if compute_uv else None,
+                    tol=tol, max_sweeps=max_sweeps, stream=stream,
+                    info_ptr=info.data_ptr() if info is not None else 0, **kw)
+    Us = [u.T for u in Ub] if compute_uv else None
+    Vs = [v.T for v in Vb] if compute_uv else None
+    return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)

@@ -1,0 +1,266 @@
+// api.cu -- the C-ABI (include/wcsvd.h): argument validation, the per-matrix planner (the W-cycle
+// level filters), workspace, descriptor upload and kernel launches.
+// Host code only; every numerical step runs in the CUDA kernels of this directory.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <vector>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "wcsvd.h"
+
+namespace wcsvd {
+namespace {
+
+constexpr int kMaxDim = 1024;
+
+double f_tb(int M, int N) { return 0.5 * N * (N - 1.0) * (8.0 * M + 6.0 * N); }
+
+// Level-0 variant for an M x N (M >= N) matrix, or 0 if it does not fit one CTA's registers.
+// Limits follow from <= 256 threads x 255 registers per CTA (l0_jacobi.cu launch_l0 table):
+// threads = (ceil(M/R) + NP/R) * G.
+int l0_variant(int M, int N) {
+  if (N <= 8) return (M / 8 + 2) * 1 <= 256 ? kL0_8 : 0;
+  if (N <= 16) return ((M + 7) / 8 + 2) * 2 <= 256 ? kL0_16 : 0;
+  if (N <= 32) {
+    if (M <= 48) return kL0_32s;
+    return ((M + 3) / 4 + 8) * 2 <= 256 ? kL0_32 : 0;
+  }
+  if (N <= 48) return ((M + 1) / 2 + 24) * 2 <= 256 ? kL0_48 : 0;
+  if (N <= 64) return ((M + 1) / 2 + 32) * 2 <= 256 ? kL0_64 : 0;
+  return 0;
+}
+
+int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
+  std::memset(p, 0, sizeof(*p));
+  p->m = m;
+  p->n = n;
+  p->swapped = (m < n) ? 1 : 0;  // iterate on A^T when m < n
+  p->M = std::max(m, n);
+  p->N = std::min(m, n);
+  p->cost = f_tb(p->M, p->N);
+  const int v = l0_variant(p->M, p->N);
+  // Alg 2 l.2: "if SVD of A^k can be implemented entirely within SM" -> Level 0.
+  if (v && (force_path == 0 || force_path == WCSVD_PATH_L0)) {
+    p->path = WCSVD_PATH_L0;
+    p->variant = v;
+    static const int np_of[] = {0, 8, 16, 32, 32, 48, 64};
+    p->n_pad = np_of[v];
+    p->m_pad = p->M;
+    return WCSVD_OK;
+  }
+  (void)force_w;
+  return WCSVD_ENOTSUP;  // Level >= 1 paths: see l1 kernels
+}
+
+struct Bucket {
+  int path, variant;
+  std::vector<int> members;  // batch indices, largest cost first
+  int maxM = 0;
+};
+
+const char* kStatus[] = {"ok", "invalid argument", "not supported", "CUDA error", "out of memory"};
+
+}  // namespace
+}  // namespace wcsvd
+
+using namespace wcsvd;
+
+extern "C" {
+
+const char* wcsvd_version(void) { return "wcsvd 0.1 sm_100a"; }
+
+const char* wcsvd_status_string(int status) {
+  if (status == WCSVD_OK) return kStatus[0];
+  if (status == WCSVD_ENOTSUP) return kStatus[2];
+  if (status == WCSVD_ECUDA) return kStatus[3];
+  if (status == WCSVD_ENOMEM) return kStatus[4];
+  if (status < 0 && status >= -12) return kStatus[1];
+  return "unknown status";
+}
+
+int wcsvd_plan(int m, int n, int force_path, int force_w, wcsvd_plan_t* out) {
+  if (m < 1) return -1;
+  if (n < 1) return -2;
+  if (!out) return -5;
+  if (m > kMaxDim || n > kMaxDim) return WCSVD_ENOTSUP;
+  return plan_one(m, n, force_path, force_w, out);
+}
+
+int wcsvd_round_robin(int np, int step, int* pairs) {
+  if (np < 2 || (np & 1) || step < 0 || step >= np - 1 || !pairs) return -1;
+  for (int k = 0; k < np / 2; ++k) {
+    const int a = rr_content(2 * k, step, np), b = rr_content(2 * k + 1, step, np);
+    pairs[2 * k] = std::min(a, b);
+    pairs[2 * k + 1] = std::max(a, b);
+  }
+  return 0;
+}
+
+static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs, size_t* off_order,
+                        size_t* off_status, size_t* off_l1) {
+  size_t off = 0;
+  auto align = [](size_t x) { return (x + 255) & ~size_t(255); };
+  *off_descs = off;
+  off = align(off + sizeof(MatDesc) * (size_t)batch);
+  *off_order = off;
+  off = align(off + sizeof(int) * (size_t)batch);
+  *off_status = off;
+  off = align(off + sizeof(int) * (size_t)batch);
+  *off_l1 = off;
+  (void)m; (void)n;
+  return off;
+}
+
+size_t wcsvd_workspace_size(int batch, const int* m, const int* n) {
+  if (batch <= 0 || !m || !n) return 0;
+  size_t a, b, c, d;
+  return ws_layout(batch, m, n, &a, &b, &c, &d);
+}
+
+int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                     double* const* S, double* const* U, double* const* V, double tol,
+                     int max_sweeps, wcsvd_stream_t stream_, const wcsvd_opts* opts) {
+  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
+  // ---- validation (nothing is enqueued on failure) ----
+  if (batch < 0) return -1;
+  if (batch == 0) return WCSVD_OK;
+  if (!m) return -2;
+  if (!n) return -3;
+  if (!A) return -4;
+  if (!lda) return -5;
+  if (!S) return -6;
+  if (opts && opts->struct_size != sizeof(wcsvd_opts)) return -12;
+  if (std::isnan(tol)) return -9;
+  const int* ldu = opts ? opts->ldu : nullptr;
+  const int* ldv = opts ? opts->ldv : nullptr;
+  for (int b = 0; b < batch; ++b) {
+    if (m[b] < 1) return -2;
+    if (n[b] < 1) return -3;
+    if (!A[b]) return -4;
+    if (lda[b] < m[b]) return -5;
+    if (!S[b]) return -6;
+    if (ldu && U && U[b] && ldu[b] < m[b]) return -12;
+    if (ldv && V && V[b] && ldv[b] < n[b]) return -12;
+  }
+  for (int b = 0; b < batch; ++b)
+    if (m[b] > kMaxDim || n[b] > kMaxDim) return WCSVD_ENOTSUP;
+
+  const int force_path = opts ? opts->force_path : 0;
+  const int force_w = opts ? opts->force_w : 0;
+  if (max_sweeps <= 0) max_sweeps = 60;
+
+  // ---- plan (a pure function of (m, n)) and bucket by kernel ----
+  std::vector<wcsvd_plan_t> plans(batch);
+  for (int b = 0; b < batch; ++b) {
+    const int rc = plan_one(m[b], n[b], force_path, force_w, &plans[b]);
+    if (rc != WCSVD_OK) return rc;
+  }
+  std::vector<Bucket> buckets;
+  for (int b = 0; b < batch; ++b) {
+    Bucket* bk = nullptr;
+    for (auto& x : buckets)
+      if (x.path == plans[b].path && x.variant == plans[b].variant) bk = &x;
+    if (!bk) {
+      buckets.push_back(Bucket{plans[b].path, plans[b].variant, {}, 0});
+      bk = &buckets.back();
+    }
+    bk->members.push_back(b);
+    bk->maxM = std::max(bk->maxM, plans[b].M);
+  }
+  for (auto& bk : buckets)
+    std::stable_sort(bk.members.begin(), bk.members.end(),
+                     [&](int x, int y) { return plans[x].cost > plans[y].cost; });
+  std::sort(buckets.begin(), buckets.end(), [&](const Bucket& x, const Bucket& y) {
+    return plans[x.members[0]].cost > plans[y.members[0]].cost;
+  });
+
+  // ---- workspace ----
+  size_t off_descs, off_order, off_status, off_l1;
+  const size_t ws_bytes = ws_layout(batch, m, n, &off_descs, &off_order, &off_status, &off_l1);
+  unsigned char* ws = nullptr;
+  bool own_ws = false;
+  if (opts && opts->workspace) {
+    if (opts->workspace_bytes < ws_bytes) return -12;
+    ws = static_cast<unsigned char*>(opts->workspace);
+  } else {
+    if (cudaMallocAsync(reinterpret_cast<void**>(&ws), ws_bytes, stream) != cudaSuccess) {
+      cudaGetLastError();
+      return WCSVD_ENOMEM;
+    }
+    own_ws = true;
+  }
+  MatDesc* d_descs = reinterpret_cast<MatDesc*>(ws + off_descs);
+  int* d_order = reinterpret_cast<int*>(ws + off_order);
+  int* d_status = reinterpret_cast<int*>(ws + off_status);
+
+  // ---- descriptors (host) -> device ----
+  std::vector<MatDesc> h(batch);
+  for (int b = 0; b < batch; ++b) {
+    const wcsvd_plan_t& p = plans[b];
+    MatDesc& d = h[b];
+    std::memset(&d, 0, sizeof(d));
+    d.A = A[b];
+    d.S = S[b];
+    d.U = U ? U[b] : nullptr;
+    d.V = V ? V[b] : nullptr;
+    d.info = opts ? opts->info : nullptr;
+    d.sweeps_inner = opts ? opts->sweeps_inner : nullptr;
+    d.m = m[b];
+    d.n = n[b];
+    d.lda = lda[b];
+    d.ldu = ldu ? ldu[b] : m[b];
+    d.ldv = ldv ? ldv[b] : n[b];
+    d.M = p.M;
+    d.N = p.N;
+    d.swapped = p.swapped;
+    d.m_pad = p.m_pad;
+    d.n_pad = p.n_pad;
+    d.w = p.w;
+    d.w2 = p.w2;
+    d.tol = (tol > 0) ? tol : std::sqrt((double)p.M) * kU53;
+    d.max_sweeps = max_sweeps;
+    d.inner_cap = (opts && opts->inner_sweeps > 0) ? opts->inner_sweeps : 1;
+    d.idx = b;
+    d.status = d_status;
+  }
+  std::vector<int> h_order;
+  h_order.reserve(batch);
+  std::vector<int> bucket_off;
+  for (auto& bk : buckets) {
+    bucket_off.push_back((int)h_order.size());
+    h_order.insert(h_order.end(), bk.members.begin(), bk.members.end());
+  }
+  cudaError_t e = cudaMemcpyAsync(d_descs, h.data(), sizeof(MatDesc) * batch, cudaMemcpyHostToDevice, stream);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d_order, h_order.data(), sizeof(int) * batch, cudaMemcpyHostToDevice, stream);
+
+  // ---- launches ----
+  for (size_t i = 0; i < buckets.size() && e == cudaSuccess; ++i) {
+    const Bucket& bk = buckets[i];
+    const int cnt = (int)bk.members.size();
+    if (bk.path == WCSVD_PATH_L0)
+      e = launch_l0(bk.variant, d_descs, d_order + bucket_off[i], cnt, bk.maxM, stream);
+    else
+      e = cudaErrorNotSupported;
+  }
+  if (e == cudaSuccess) e = launch_complete(d_descs, batch, stream);
+  if (own_ws) cudaFreeAsync(ws, stream);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ECUDA;
+  }
+  return WCSVD_OK;
+}
+
+int wcsvd_batched(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                  double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
+                  wcsvd_stream_t stream) {
+  return wcsvd_batched_ex(batch, m, n, A, lda, S, U, V, tol, max_sweeps, stream, nullptr);
+}
+
+}  // extern "C"

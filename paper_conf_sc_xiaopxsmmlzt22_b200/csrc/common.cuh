@@ -1,0 +1,75 @@
+// common.cuh -- shared definitions of the CUDA path (kernels, planner, C-ABI). No oracle code.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "wcsvd.h"
+
+#define WCSVD_HD __host__ __device__ __forceinline__
+
+namespace wcsvd {
+
+constexpr double kU53 = 1.1102230246251565404e-16;  // 2^-53, fp64 unit roundoff
+
+// ---------------------------------------------------------------------------------------------
+// Round-robin (circle method) schedule, in "slot" form (§II.B; §IV.C).
+// np slots hold the np indices; at every step the pairs are the fixed slot pairs (2k, 2k+1):
+// top[k] = slot 2k, bot[k] = slot 2k+1. Between steps the contents move along one ring:
+//   top[1] -> top[2] -> ... -> top[h-1] -> bot[h-1] -> bot[h-2] -> ... -> bot[0] -> top[1],
+// with top[0] fixed (h = np/2). After np-1 steps every pair has met exactly once and every index
+// is back in its own slot, so at sweep boundaries slot j holds original index j. Keeping pairs at
+// fixed slots lets register-resident kernels use static register indices (the move is a rename).
+// ---------------------------------------------------------------------------------------------
+WCSVD_HD int rr_ring_index(int slot, int np) {  // position on the ring; -1 for the fixed slot 0
+  const int h = np >> 1;
+  if (slot == 0) return -1;
+  const int k = slot >> 1;
+  return (slot & 1) ? (2 * h - 2 - k) : (k - 1);
+}
+WCSVD_HD int rr_slot_of_ring(int r, int np) {
+  const int h = np >> 1;
+  return (r <= h - 2) ? 2 * (r + 1) : 2 * (2 * h - 2 - r) + 1;
+}
+// Slot a value in `slot` moves to after one step.
+WCSVD_HD int rr_dest(int slot, int np) {
+  if (slot == 0 || np == 2) return slot;
+  const int L = np - 1;
+  int r = rr_ring_index(slot, np) + 1;
+  if (r == L) r = 0;
+  return rr_slot_of_ring(r, np);
+}
+// Original index held by `slot` at step s (0 <= s < np-1).
+WCSVD_HD int rr_content(int slot, int s, int np) {
+  if (slot == 0 || np == 2) return slot;
+  const int L = np - 1;
+  int r = rr_ring_index(slot, np) - s;
+  r %= L;
+  if (r < 0) r += L;
+  return rr_slot_of_ring(r, np);
+}
+
+// Per-matrix descriptor, built on the host by the planner and copied to the device.
+struct MatDesc {
+  const double* A;
+  double* S;
+  double* U;
+  double* V;
+  int* info;
+  int* sweeps_inner;
+  double* W;   // Level >= 1 working copy (m_pad x n_pad, ld m_pad), or nullptr
+  double* Vw;  // Level >= 1 V accumulator (n_pad x n_pad, ld n_pad), or nullptr
+  double tol;
+  int m, n, lda, ldu, ldv;
+  int M, N, swapped;
+  int m_pad, n_pad, w, w2;
+  int max_sweeps, inner_cap;
+  int idx;      // index of this matrix in the caller's batch (info / status arrays)
+  int* status;  // internal per-matrix status flags (workspace), e.g. kNeedsCompletion
+};
+
+// Status flags a kernel can leave for the completion pass (Z14): bit 0 = some sigma_j below the
+// rank threshold; those U columns were written as 0 and need the deterministic MGS completion.
+constexpr int kNeedsCompletion = 1;
+
+}  // namespace wcsvd

@@ -1,0 +1,26 @@
+// kernels.h -- launchers of the CUDA path (internal).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace wcsvd {
+
+// Level-0 kernel variants (NP = padded columns, G column groups, R rows per thread).
+enum L0Variant {
+  kL0_8 = 1,    // NP=8,  G=1, R=8
+  kL0_16 = 2,   // NP=16, G=2, R=8
+  kL0_32 = 3,   // NP=32, G=2, R=4
+  kL0_32s = 4,  // NP=32, G=2, R=1 (latency-bound small batches)
+  kL0_48 = 5,   // NP=48, G=2, R=2
+  kL0_64 = 6,   // NP=64, G=2, R=2
+};
+
+cudaError_t launch_l0(int variant, const MatDesc* descs, const int* order, int count, int maxM,
+                      cudaStream_t stream);
+
+}  // namespace wcsvd
+
+namespace wcsvd {
+cudaError_t launch_complete(const MatDesc* descs, int count, cudaStream_t stream);
+}  // namespace wcsvd

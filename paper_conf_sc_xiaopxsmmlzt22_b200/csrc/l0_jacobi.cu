@@ -1,0 +1,442 @@
+// l0_jacobi.cu -- Level-0 batched SVD kernel: the whole one-sided Jacobi of a matrix that fits
+// on-chip, in one CTA, with every sweep in-kernel and finalisation fused
+// (Alg 2 l.2-3; Step 1; kernel design §IV.B).
+//
+// B200 design. The paper keeps the matrix in shared memory and gives each column
+// pair an alpha-warp. On sm_100a an SMEM-resident sweep is bound by the 128 B/clk
+// shared-memory port (every element is read and written once per step), so here the working
+// matrix X (M x NP) and V (NP x NP) live in REGISTERS, distributed by rows: a thread holds R rows
+// x NL = NP/G columns; G adjacent lanes share one row-group. The round-robin pairs always sit in
+// fixed slot pairs (2k, 2k+1) (common.cuh), so a rotation's outputs are written straight into the
+// registers of their destination slots (the column permutation is a register rename, ping-ponged
+// between two arrays); only the two ring elements that cross a column-group boundary move, by one
+// warp shuffle each. Per step the cross-row work is one fixed-order reduction of the partial dot
+// products gamma_k = sum_r x_r,2k x_r,2k+1 (through SMEM, by one warp: lane k owns pair k) and
+// one broadcast of (c_k, s_k). Norms a_i^T a_i are cached and updated by eq (6)
+// in its closed form alpha' = alpha + t gamma, beta' = beta - t gamma
+// (identical, since t^2 + 2 tau t - 1 = 0); they are recomputed exactly at the first step of every
+// sweep; sigma is recomputed exactly at finalisation.
+#include <cuda_runtime.h>
+
+#include <cmath>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace wcsvd {
+
+namespace {
+
+// Rotation of eq (4) for squared norms alpha, beta and dot product gamma, with the
+// threshold test of SURVEY Z5/Z6. tau = (alpha - beta)/(2 gamma) and
+// t = sgn(tau)/(|tau| + sqrt(1 + tau^2)) are evaluated as t = sgn(tau) 2|gamma| / (|d| + sqrt(d^2 +
+// 4 gamma^2)), d = alpha - beta (the same number, multiplied through by 2|gamma|; one division
+// instead of three). sgn(0) = +1 (Z4). Valid while d^2 + 4 gamma^2 does not overflow (column norms
+// below ~1e150). Returns true (and c, s, t) if the pair rotates.
+__device__ __forceinline__ bool jacobi_rot(double alpha, double beta, double gamma, double tol,
+                                           double& c, double& s, double& t) {
+  c = 1.0; s = 0.0; t = 0.0;
+  if (alpha == 0.0 || beta == 0.0) return false;
+  if (fabs(gamma) <= tol * (sqrt(alpha) * sqrt(beta))) return false;
+  const double d = alpha - beta;
+  const double r = sqrt(fma(d, d, 4.0 * gamma * gamma));
+  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 1.0 : -1.0;  // sgn(tau)
+  t = sg * (2.0 * fabs(gamma)) / (fabs(d) + r);
+  c = rsqrt(fma(t, t, 1.0));  // c = 1/sqrt(1+t^2)
+  s = t * c;                  // s = t c
+  return true;
+}
+
+// Per-CTA state shared by the step functions.
+struct L0Ctx {
+  double* part_g;  // [RW][PS] partial gamma per (row-thread, pair)
+  double* part_a;  // [RW][PS] partial alpha (first step of a sweep)
+  double* part_b;  // [RW][PS] partial beta
+  double* nrm;     // [2][NP]  cached squared norms per slot, double-buffered by step parity
+  double2* cs;     // [G][LP+1] (c, s) per pair, padded against bank conflicts
+  int* flags;      // [0],[1] rotation flag per sweep parity; [2] non-finite; [3] completion
+  int RW, PS;
+  int tid, g, rt;
+  bool isW;
+  int dtop, dbot;  // reducer lane k: slots that the contents of slots 2k, 2k+1 move to
+  double tol;
+  int gs;          // global step counter
+  int sweep;       // completed sweeps
+};
+
+// One round-robin step: every pair of the matrix is orthogonalised once; reads the
+// slots from x, writes the rotated, moved slots to y.
+template <int NP, int G, int R, bool FIRST>
+__device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
+                                        double (&y)[R][NP / G]) {
+  constexpr int NL = NP / G;
+  constexpr int LP = NL / 2;
+  constexpr int NPAIR = NP / 2;
+  static_assert(LP >= 2 && NPAIR <= 32, "L0 tile");
+  const int g = cx.g;
+  // Phase 1: this thread's partial dot products for its pairs (and squared norms at sweep start).
+  if (cx.isW) {
+    const int base = cx.rt * cx.PS + g * LP;
+#pragma unroll
+    for (int j = 0; j < LP; ++j) {
+      double gm = 0.0, al = 0.0, be = 0.0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        gm = fma(x[r][2 * j], x[r][2 * j + 1], gm);
+        if (FIRST) {
+          al = fma(x[r][2 * j], x[r][2 * j], al);
+          be = fma(x[r][2 * j + 1], x[r][2 * j + 1], be);
+        }
+      }
+      cx.part_g[base + j] = gm;
+      if (FIRST) {
+        cx.part_a[base + j] = al;
+        cx.part_b[base + j] = be;
+      }
+    }
+  }
+  __syncthreads();
+  // Phase 2 (warp 0, lane k = pair k): fixed-order sum over row-threads, eq (4), eq (6).
+  if (cx.tid < 32) {
+    if (FIRST && cx.tid == 0) cx.flags[(cx.sweep + 1) & 1] = 0;
+    const int k = cx.tid;
+    if (k < NPAIR) {
+      const int PS = cx.PS, RW = cx.RW;
+      double g4[4] = {0.0, 0.0, 0.0, 0.0}, a4[4] = {0.0, 0.0, 0.0, 0.0}, b4[4] = {0.0, 0.0, 0.0, 0.0};
+      // rows [RW, RW4) of the partial arrays are zero (set once at kernel start)
+      for (int i = 0; i < RW; i += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          g4[u] += cx.part_g[(i + u) * PS + k];
+          if (FIRST) {
+            a4[u] += cx.part_a[(i + u) * PS + k];
+            b4[u] += cx.part_b[(i + u) * PS + k];
+          }
+        }
+      }
+      const double gm = (g4[0] + g4[1]) + (g4[2] + g4[3]);
+      const int cur = cx.gs & 1;
+      double al, be;
+      if (FIRST) {
+        al = (a4[0] + a4[1]) + (a4[2] + a4[3]);
+        be = (b4[0] + b4[1]) + (b4[2] + b4[3]);
+      } else {
+        al = cx.nrm[cur * NP + 2 * k];
+        be = cx.nrm[cur * NP + 2 * k + 1];
+      }
+      double c, s, t;
+      const bool rot = jacobi_rot(al, be, gm, cx.tol, c, s, t);
+      cx.cs[(k / LP) * (LP + 1) + (k % LP)] = make_double2(c, s);
+      cx.nrm[(cur ^ 1) * NP + cx.dtop] = rot ? fma(t, gm, al) : al;
+      cx.nrm[(cur ^ 1) * NP + cx.dbot] = rot ? fma(-t, gm, be) : be;
+      if (rot) cx.flags[cx.sweep & 1] = 1;
+    }
+  }
+  __syncthreads();
+  // Phase 3: rotate this thread's rows of X or V (eq 3) and move the slots (common.cuh ring).
+  // Outputs of local pair j: top -> top[j+1], bot -> bot[j-1]. Group 0 keeps top[0] and sends
+  // bot[0] to its top[1]; other groups receive top[0] from the left neighbour lane; the last group
+  // moves its last top to its last bot, the others receive their last bot from the right.
+  double top0[R], send_l[R], send_r[R];
+  const double2* cs = cx.cs + g * (LP + 1);
+#pragma unroll
+  for (int j = 0; j < LP; ++j) {
+    const double2 p = cs[j];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const double a = x[r][2 * j], b = x[r][2 * j + 1];
+      // eq (3): (a^_i, a^_j) = (a_i, a_j) [[c, -s], [s, c]]
+      const double na = fma(p.y, b, p.x * a);
+      const double nb = fma(-p.y, a, p.x * b);
+      if (j == 0) top0[r] = na;
+      else if (j + 1 < LP) y[r][2 * (j + 1)] = na;
+      else send_r[r] = na;
+      if (j == 0) send_l[r] = nb;
+      else y[r][2 * (j - 1) + 1] = nb;
+    }
+  }
+  const bool gfirst = (g == 0), glast = (g == G - 1);
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    double from_left = 0.0, from_right = 0.0;
+    if (G > 1) {
+      from_left = __shfl_up_sync(0xffffffffu, send_r[r], 1);
+      from_right = __shfl_down_sync(0xffffffffu, send_l[r], 1);
+    }
+    y[r][0] = gfirst ? top0[r] : from_left;
+    y[r][2] = gfirst ? send_l[r] : top0[r];
+    y[r][2 * (LP - 1) + 1] = glast ? send_r[r] : from_right;
+  }
+  ++cx.gs;
+}
+
+// One sweep of NP-1 steps starting in x; ends in y with every slot back in its original column.
+template <int NP, int G, int R>
+__device__ __forceinline__ void l0_sweep(L0Ctx& cx, double (&x)[R][NP / G], double (&y)[R][NP / G]) {
+  l0_step<NP, G, R, true>(cx, x, y);
+  for (int i = 0; i < (NP - 2) / 2; ++i) {
+    l0_step<NP, G, R, false>(cx, y, x);
+    l0_step<NP, G, R, false>(cx, x, y);
+  }
+}
+
+}  // namespace
+
+// Shared-memory bytes of one CTA (must match the carve-up in the kernel).
+template <int NP, int G, int R>
+size_t l0_smem_bytes(int M) {
+  const int RW = ((M + R - 1) / R + 3) / 4 * 4;
+  const int PS = NP / 2 + 1;
+  const int RV = NP / R;
+  const int LP = NP / G / 2;
+  return sizeof(double2) * G * (LP + 1) + sizeof(double) * (2 * NP + 2 * NP + (size_t)RV * NP) +
+         sizeof(double) * 3 * (size_t)RW * PS + sizeof(int) * (NP + 8);
+}
+
+// One CTA per matrix. Thread t: group g = t % G, row-thread rt = t / G. Row-threads [0, RW) hold
+// rows rt*R .. rt*R+R-1 of X; row-threads [RW, RW+RV) hold rows of V (RV = NP/R); the rest (to a
+// multiple of 32) hold zeros and only take part in shuffles.
+template <int NP, int G, int R, int MAXT>
+__global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restrict__ descs,
+                                                        const int* __restrict__ order) {
+  constexpr int NL = NP / G;
+  constexpr int LP = NL / 2;
+  constexpr int NPAIR = NP / 2;
+  constexpr int RV = NP / R;
+  const MatDesc d = descs[order[blockIdx.x]];
+  const int M = d.M, N = d.N;
+  const int RW = (M + R - 1) / R;
+  const int PS = NPAIR + 1;  // odd stride (doubles): conflict-free partial writes and reads
+  const int T = blockDim.x;
+  const int tid = threadIdx.x;
+  const int g = tid % G;
+  const int rt = tid / G;
+  const bool isW = rt < RW;
+  const bool isV = !isW && rt < RW + RV;
+
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  double2* s_cs = reinterpret_cast<double2*>(smem_raw);  // [G][LP+1]
+  double* s_nrm = reinterpret_cast<double*>(s_cs + G * (LP + 1));  // [2][NP]
+  double* s_sig = s_nrm + 2 * NP;                        // [NP]
+  double* s_sgn = s_sig + NP;                            // [NP]
+  double* s_vbest = s_sgn + NP;                          // [RV][NP]
+  const int RW4 = (RW + 3) / 4 * 4;                      // partial rows padded to 4 (zeros)
+  double* s_part = s_vbest + RV * NP;                    // [3][RW4][PS]
+  int* s_rank = reinterpret_cast<int*>(s_part + 3 * RW4 * PS);  // [NP]
+  int* s_flags = s_rank + NP;                            // [8]
+  if (tid < 8) s_flags[tid] = 0;
+  for (int e = tid; e < 3 * RW4 * PS; e += T) s_part[e] = 0.0;
+  __syncthreads();
+
+  // ---- Stage-in: X = A (m >= n) or A^T (m < n), zero-padded; V = I. ----
+  double xa[R][NL], xb[R][NL];
+  bool bad = false;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+      const int col = g * NL + l;
+      double v = 0.0;
+      if (isW) {
+        const int row = rt * R + r;
+        if (row < M && col < N) {
+          v = d.swapped ? d.A[(size_t)row * d.lda + col] : d.A[(size_t)col * d.lda + row];
+          bad |= !isfinite(v);
+        }
+      } else if (isV) {
+        v = ((rt - RW) * R + r == col) ? 1.0 : 0.0;
+      }
+      xa[r][l] = v;
+    }
+  }
+  if (bad) atomicOr(&s_flags[2], 1);
+  __syncthreads();
+  const bool nonfinite = s_flags[2] != 0;
+
+  L0Ctx cx;
+  cx.part_g = s_part;
+  cx.part_a = s_part + RW4 * PS;
+  cx.part_b = s_part + 2 * RW4 * PS;
+  cx.nrm = s_nrm;
+  cx.cs = s_cs;
+  cx.flags = s_flags;
+  cx.RW = RW;
+  cx.PS = PS;
+  cx.tid = tid;
+  cx.g = g;
+  cx.rt = rt;
+  cx.isW = isW;
+  cx.dtop = rr_dest(2 * (tid % 32), NP);
+  cx.dbot = rr_dest(2 * (tid % 32) + 1, NP);
+  cx.tol = d.tol;
+  cx.gs = 0;
+  cx.sweep = 0;
+  bool converged = false;
+  bool in_b = false;
+  if (!nonfinite) {
+    for (;;) {
+      l0_sweep<NP, G, R>(cx, xa, xb);  // ends in xb
+      ++cx.sweep;
+      if (s_flags[(cx.sweep - 1) & 1] == 0) { converged = true; in_b = true; break; }
+      if (cx.sweep >= d.max_sweeps) { in_b = true; break; }
+      l0_sweep<NP, G, R>(cx, xb, xa);  // ends in xa
+      ++cx.sweep;
+      if (s_flags[(cx.sweep - 1) & 1] == 0) { converged = true; break; }
+      if (cx.sweep >= d.max_sweeps) break;
+    }
+  }
+  const int sweep = cx.sweep;
+  if (in_b) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int l = 0; l < NL; ++l) xa[r][l] = xb[r][l];
+  }
+
+  // ---- Finalisation: sigma_j = ||x_j|| (fresh, fixed order), stable descending
+  // rank (Z15), U = X / sigma, sign rule on the square factor V_x (Z15), un-orientation.
+  __syncthreads();
+  if (isW) {
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+      double a = 0.0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) a = fma(xa[r][l], xa[r][l], a);
+      const int col = g * NL + l;  // [RW][NP] view over the first two partial sections
+      s_part[(col < NPAIR ? 0 : RW4) * PS + rt * PS + (col % NPAIR)] = a;
+    }
+  }
+  if (isV) {
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+      double best = 0.0;
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (fabs(xa[r][l]) > fabs(best)) best = xa[r][l];
+      s_vbest[(rt - RW) * NP + g * NL + l] = best;
+    }
+  }
+  __syncthreads();
+  for (int j = tid; j < NP; j += T) {
+    const int base = (j < NPAIR ? 0 : RW4) * PS + (j % NPAIR);
+    double a4[4] = {0.0, 0.0, 0.0, 0.0};
+    for (int i = 0; i < RW; i += 4) {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) a4[u] += s_part[base + (i + u) * PS];
+    }
+    s_sig[j] = sqrt((a4[0] + a4[1]) + (a4[2] + a4[3]));
+    double best = 0.0;
+    for (int i = 0; i < RV; ++i) {
+      const double v = s_vbest[i * NP + j];
+      if (fabs(v) > fabs(best)) best = v;
+    }
+    s_sgn[j] = (best < 0.0) ? -1.0 : 1.0;
+  }
+  __syncthreads();
+  for (int j = tid; j < NP; j += T) {
+    int rk = -1;
+    if (j < N && nonfinite) {
+      rk = j;  // NaN sigmas: identity order, every column written
+    } else if (j < N) {
+      rk = 0;
+      const double sj = s_sig[j];
+      for (int i = 0; i < N; ++i) {
+        const double si = s_sig[i];
+        rk += (si > sj) || (si == sj && i < j);
+      }
+    }
+    s_rank[j] = rk;
+  }
+  __syncthreads();
+  double sig1 = 0.0;
+  for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
+  const double thresh = sig1 * (double)M * kU53;  // Z14 rank threshold
+  const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
+  // X-space factors: U_w -> U (V if swapped), V_x -> V (U if swapped).
+  double* dstW = d.swapped ? d.V : d.U;
+  const int ldW = d.swapped ? d.ldv : d.ldu;
+  double* dstV = d.swapped ? d.U : d.V;
+  const int ldV = d.swapped ? d.ldu : d.ldv;
+  bool needs_completion = false;
+  if (isW && dstW) {
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+      const int col = g * NL + l;
+      if (col < N) {
+        const int rk = s_rank[col];
+        const double sj = s_sig[col];
+        const double sgn = s_sgn[col];
+        const bool ok = sj > thresh;
+        needs_completion |= !ok;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int row = rt * R + r;
+          if (row < M)  // rank-deficient columns: signed zero, completed by complete_u_kernel
+            dstW[(size_t)rk * ldW + row] = nonfinite ? nanv : (ok ? sgn * (xa[r][l] / sj) : sgn * 0.0);
+        }
+      }
+    }
+  }
+  if (isV && dstV) {
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+      const int col = g * NL + l;
+      if (col < N) {
+        const int rk = s_rank[col];
+        const double sgn = s_sgn[col];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int vrow = (rt - RW) * R + r;
+          if (vrow < N) dstV[(size_t)rk * ldV + vrow] = nonfinite ? nanv : sgn * xa[r][l];
+        }
+      }
+    }
+  }
+  if (needs_completion && !nonfinite) atomicOr(&s_flags[3], 1);
+  for (int j = tid; j < N; j += T) d.S[s_rank[j]] = nonfinite ? nanv : s_sig[j];
+  __syncthreads();
+  if (tid == 0) {
+    if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
+    if (d.sweeps_inner) d.sweeps_inner[d.idx] = 0;
+    if (d.status) d.status[d.idx] = (s_flags[3] && dstW) ? kNeedsCompletion : 0;
+  }
+}
+
+// ---- launcher ----
+template <int NP, int G, int R, int MAXT>
+static cudaError_t launch_l0_t(const MatDesc* descs, const int* order, int count, int maxM,
+                               cudaStream_t stream) {
+  const int RW = (maxM + R - 1) / R;
+  int threads = (RW + NP / R) * G;
+  threads = (threads + 31) / 32 * 32;
+  if (threads > MAXT) return cudaErrorInvalidConfiguration;
+  const size_t smem = l0_smem_bytes<NP, G, R>(maxM);
+  auto kern = l0_jacobi_kernel<NP, G, R, MAXT>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  kern<<<count, threads, smem, stream>>>(descs, order);
+  return cudaGetLastError();
+}
+
+int l0_max_threads(int variant) {
+  switch (variant) {
+    case kL0_32s: return 512;
+    default: return 256;
+  }
+}
+
+// Variant table (planner ids). E = R * NP / G doubles per thread.
+cudaError_t launch_l0(int variant, const MatDesc* descs, const int* order, int count, int maxM,
+                      cudaStream_t stream) {
+  switch (variant) {
+    case kL0_8:   return launch_l0_t<8, 1, 8, 256>(descs, order, count, maxM, stream);
+    case kL0_16:  return launch_l0_t<16, 2, 8, 256>(descs, order, count, maxM, stream);
+    case kL0_32:  return launch_l0_t<32, 2, 4, 256>(descs, order, count, maxM, stream);
+    case kL0_32s: return launch_l0_t<32, 2, 1, 512>(descs, order, count, maxM, stream);
+    case kL0_48:  return launch_l0_t<48, 2, 2, 256>(descs, order, count, maxM, stream);
+    case kL0_64:  return launch_l0_t<64, 4, 4, 256>(descs, order, count, maxM, stream);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace wcsvd

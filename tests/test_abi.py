@@ -1,0 +1,84 @@
+"""Host-side checks of the C-ABI library (no GPU needed): it loads, exports every symbol that
+include/wcsvd.h declares, validates arguments without enqueuing, and its planner / schedule are
+pure functions of (m, n) with the round-robin properties of PAPER.md:64 and PAPER.md:253."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_sc_xiaopxsmmlzt22_b200 as wc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared_symbols():
+    src = open(os.path.join(ROOT, "include", "wcsvd.h")).read()
+    return sorted(set(re.findall(r"WCSVD_API\s+[\w\s\*]+?\b(wcsvd_\w+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    L = wc.lib()
+    syms = _declared_symbols()
+    assert len(syms) >= 7
+    for s in syms:
+        assert hasattr(L, s), s
+    assert b"sm_100a" in L.wcsvd_version()
+
+
+def test_status_strings():
+    L = wc.lib()
+    assert L.wcsvd_status_string(0) == b"ok"
+    assert L.wcsvd_status_string(-100) == b"not supported"
+    assert L.wcsvd_status_string(-3) == b"invalid argument"
+
+
+def test_argument_validation_is_synchronous_and_enqueues_nothing():
+    L = wc.lib()
+    one = np.array([4], dtype=np.int32)
+    bad_m = np.array([0], dtype=np.int32)
+    ptr = np.array([8], dtype=np.uint64)  # never dereferenced: validation fails first
+    lda3 = np.array([3], dtype=np.int32)
+    P = lambda a: a.ctypes.data
+    assert L.wcsvd_batched(-1, None, None, None, None, None, None, None, 0.0, 0, None) == -1
+    assert L.wcsvd_batched(0, None, None, None, None, None, None, None, 0.0, 0, None) == 0
+    assert L.wcsvd_batched(1, P(bad_m), P(one), P(ptr), P(one), P(ptr), None, None, 0.0, 0, None) == -2
+    assert L.wcsvd_batched(1, P(one), P(bad_m), P(ptr), P(one), P(ptr), None, None, 0.0, 0, None) == -3
+    assert L.wcsvd_batched(1, P(one), P(one), None, P(one), P(ptr), None, None, 0.0, 0, None) == -4
+    assert L.wcsvd_batched(1, P(one), P(one), P(ptr), P(lda3), P(ptr), None, None, 0.0, 0, None) == -5
+    assert L.wcsvd_batched(1, P(one), P(one), P(ptr), P(one), None, None, None, 0.0, 0, None) == -6
+    big = np.array([1025], dtype=np.int32)
+    assert L.wcsvd_batched(1, P(big), P(one), P(ptr), P(big), P(ptr), None, None, 0.0, 0, None) == -100
+    assert L.wcsvd_batched(1, P(one), P(one), P(ptr), P(one), P(ptr), None, None, float("nan"), 0, None) == -9
+
+
+def test_workspace_size_positive():
+    m = np.array([64, 256, 1024], dtype=np.int32)
+    n = np.array([64, 256, 1000], dtype=np.int32)
+    assert wc.lib().wcsvd_workspace_size(3, m.ctypes.data, n.ctypes.data) > 0
+
+
+@pytest.mark.parametrize("np_", [2, 4, 6, 8, 16, 32, 48, 64, 128, 256])
+def test_round_robin_covers_every_pair_once(np_):
+    # P5: np-1 steps x np/2 disjoint pairs cover all np(np-1)/2 pairs exactly once.
+    seen = set()
+    for s in range(np_ - 1):
+        pairs = wc.round_robin(np_, s)
+        idx = [i for p in pairs for i in p]
+        assert sorted(idx) == list(range(np_))  # each index once per step
+        for p in pairs:
+            assert p[0] < p[1] and p not in seen
+            seen.add(p)
+    assert len(seen) == np_ * (np_ - 1) // 2
+
+
+def test_plan_is_pure_and_transposes_wide():
+    p1 = wc.plan(40, 24)
+    p2 = wc.plan(24, 40)
+    assert p1["swapped"] == 0 and p2["swapped"] == 1
+    assert (p1["M"], p1["N"]) == (p2["M"], p2["N"]) == (40, 24)
+    assert p1["path"] == p2["path"] == wc.PATH_L0
+    assert wc.plan(40, 24) == p1
+    for (m, n) in [(32, 32), (64, 64)]:
+        assert wc.plan(m, n)["path"] == wc.PATH_L0
