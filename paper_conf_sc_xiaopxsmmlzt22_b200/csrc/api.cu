@@ -53,8 +53,24 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
     p->m_pad = p->M;
     return WCSVD_OK;
   }
-  (void)force_w;
-  return WCSVD_ENOTSUP;  // Level >= 1 paths: see l1 kernels
+  if (force_path == WCSVD_PATH_L0) return WCSVD_ENOTSUP;
+  // Alg 2 l.5-11: Level 1, column blocks of width w; the pair Gram's EVD runs on-chip.
+  int w = (p->N <= 96) ? 8 : 16;
+  if (force_w == 8 || force_w == 16) w = force_w;
+  else if (force_w != 0) return WCSVD_ENOTSUP;
+  p->path = WCSVD_PATH_GRAM;
+  p->w = w;
+  p->n_pad = (p->N + 2 * w - 1) / (2 * w) * (2 * w);
+  p->m_pad = (p->M + 15) / 16 * 16;
+  const int pairs = p->n_pad / w / 2;
+  p->variant = (w == 8) ? kL1_16x4 : (pairs >= 8 ? kL1_32x8 : kL1_32x4);
+  return WCSVD_OK;
+}
+
+size_t l1_bytes(const wcsvd_plan_t& p) {
+  if (p.path == WCSVD_PATH_L0) return 0;
+  const size_t b = sizeof(double) * ((size_t)p.m_pad * p.n_pad + (size_t)p.n_pad * p.n_pad);
+  return (b + 255) & ~size_t(255);
 }
 
 struct Bucket {
@@ -102,7 +118,8 @@ int wcsvd_round_robin(int np, int step, int* pairs) {
 }
 
 static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs, size_t* off_order,
-                        size_t* off_status, size_t* off_l1) {
+                        size_t* off_status, size_t* off_l1, std::vector<size_t>* l1_off = nullptr,
+                        int force_path = 0, int force_w = 0) {
   size_t off = 0;
   auto align = [](size_t x) { return (x + 255) & ~size_t(255); };
   *off_descs = off;
@@ -112,7 +129,14 @@ static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs
   *off_status = off;
   off = align(off + sizeof(int) * (size_t)batch);
   *off_l1 = off;
-  (void)m; (void)n;
+  if (l1_off) l1_off->assign(batch, 0);
+  for (int b = 0; b < batch; ++b) {
+    wcsvd_plan_t p;
+    if (m[b] < 1 || n[b] < 1 || m[b] > kMaxDim || n[b] > kMaxDim) continue;
+    if (plan_one(m[b], n[b], force_path, force_w, &p) != WCSVD_OK) continue;
+    if (l1_off) (*l1_off)[b] = off;
+    off += l1_bytes(p);
+  }
   return off;
 }
 
@@ -181,7 +205,9 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
 
   // ---- workspace ----
   size_t off_descs, off_order, off_status, off_l1;
-  const size_t ws_bytes = ws_layout(batch, m, n, &off_descs, &off_order, &off_status, &off_l1);
+  std::vector<size_t> l1_off;
+  const size_t ws_bytes =
+      ws_layout(batch, m, n, &off_descs, &off_order, &off_status, &off_l1, &l1_off, force_path, force_w);
   unsigned char* ws = nullptr;
   bool own_ws = false;
   if (opts && opts->workspace) {
@@ -227,6 +253,10 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     d.inner_cap = (opts && opts->inner_sweeps > 0) ? opts->inner_sweeps : 1;
     d.idx = b;
     d.status = d_status;
+    if (p.path != WCSVD_PATH_L0) {
+      d.W = reinterpret_cast<double*>(ws + l1_off[b]);
+      d.Vw = d.W + (size_t)p.m_pad * p.n_pad;
+    }
   }
   std::vector<int> h_order;
   h_order.reserve(batch);
@@ -246,7 +276,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     if (bk.path == WCSVD_PATH_L0)
       e = launch_l0(bk.variant, d_descs, d_order + bucket_off[i], cnt, bk.maxM, stream);
     else
-      e = cudaErrorNotSupported;
+      e = launch_l1(bk.variant, d_descs, d_order + bucket_off[i], cnt, stream);
   }
   if (e == cudaSuccess) e = launch_complete(d_descs, batch, stream);
   if (own_ws) cudaFreeAsync(ws, stream);

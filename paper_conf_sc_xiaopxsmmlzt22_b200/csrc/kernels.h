@@ -16,6 +16,15 @@ enum L0Variant {
   kL0_64 = 6,   // NP=64, G=2, R=2
 };
 
+// Level-1 Gram-path variants (pair panel width 2w, warps per CTA).
+enum L1Variant {
+  kL1_16x4 = 11,  // 2w = 16, 4 warps
+  kL1_32x4 = 12,  // 2w = 32, 4 warps
+  kL1_32x8 = 13,  // 2w = 32, 8 warps
+};
+
+cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
+
 cudaError_t launch_l0(int variant, const MatDesc* descs, const int* order, int count, int maxM,
                       cudaStream_t stream);
 

@@ -1,0 +1,491 @@
+// l1_gram.cu -- Level-1 block one-sided Jacobi over column-block pairs, Gram path:
+// (1) Gram B_ij = A_ij^T A_ij, (2) threshold Jacobi EVD of B_ij in shared memory / registers,
+// (3) GEMM update A_ij <- A_ij J_ij and V_ij <- V_ij J_ij, (4) off-norm test -- Alg 1 l.5-7
+// (PAPER.md:68-70), Alg 2 l.10-11 + l.16, Step 2, the parallel
+// EVD of §IV.C and the two batched GEMMs of §IV.D.
+//
+// B200 design: one CTA per matrix runs every sweep in-kernel (no host round
+// trip); each warp owns one column-block pair of the current round-robin step at a
+// time; a CTA barrier separates steps. The working copy W (m_pad x n_pad) and V live in global
+// memory (L2-resident while the CTA works on them). Both contractions use FP64 DMMA.8x8x4 tiles
+// fed straight from L2 into registers (no SMEM staging needed: each fragment load is 8 columns x
+// 32 contiguous bytes); the Gram computes only the upper tiles. The EVD is the paper's parallel
+// two-sided Jacobi with round-robin pairs: B stays in SMEM in original index
+// order and is updated in 2x2 quads; J is accumulated in registers (row x of J in lane x) in
+// "slot" order so that every rotation writes fixed registers (common.cuh). Threshold rotations make
+// J = I exactly once B is diagonal to tol; the EVD is capped at inner_cap sweeps
+// (Z8); J is re-orthogonalised by one Newton-Schulz step J <- J - J (J^T J - I)/2 before it is
+// applied (Z9(ii)). A pair whose Gram is already diagonal to tol is skipped with no writes; a
+// sweep in which every pair is skipped ends the iteration (Z6, Z9(iii)).
+#include <cuda_runtime.h>
+
+#include <cmath>
+
+#include "common.cuh"
+#include "dmma.cuh"
+#include "kernels.h"
+
+namespace wcsvd {
+
+namespace {
+
+__device__ __forceinline__ bool rot_params(double alpha, double beta, double gamma, double tol,
+                                           double& c, double& s, double& t) {
+  // eq (4) / §II.D rho with the threshold of SURVEY Z5/Z6; see l0_jacobi.cu.
+  c = 1.0; s = 0.0; t = 0.0;
+  if (alpha <= 0.0 || beta <= 0.0) return false;
+  if (fabs(gamma) <= tol * (sqrt(alpha) * sqrt(beta))) return false;
+  const double d = alpha - beta;
+  const double r = sqrt(fma(d, d, 4.0 * gamma * gamma));
+  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 1.0 : -1.0;
+  t = sg * (2.0 * fabs(gamma)) / (fabs(d) + r);
+  c = rsqrt(fma(t, t, 1.0));
+  s = t * c;
+  return true;
+}
+
+template <int W2>
+struct PairCfg {
+  static constexpr int W = W2 / 2;          // block width w
+  static constexpr int CG = W2 / 8;         // 8-column groups per pair panel
+  static constexpr int NTU = CG * (CG + 1) / 2;  // upper tiles of the 2w x 2w Gram
+  static constexpr int BS = W2 + 1;         // SMEM row stride of 2w x 2w buffers (doubles)
+  static constexpr int NPR = W2 / 2;        // rotation pairs per EVD step
+  static constexpr int LPK = 32 / NPR;      // lanes per row-pair k in the quad phase
+  static constexpr int QPL = NPR / LPK;     // quads per lane
+  static_assert(W2 == 16 || W2 == 32, "pair panel width");
+};
+
+// Per-warp SMEM region.
+template <int W2>
+struct WarpSmem {
+  double* B;    // [W2][BS] Gram / E = J^T J - I / J'
+  double* S;    // [W2][BS] staged J
+  double2* cs;  // [NPR]    (c, s) of the step's rotations
+  double* tt;   // [NPR]    t of the step's rotations (0 = none)
+  int2* pq;     // [NPR]    (p, q) original indices of the step's pairs
+  __host__ __device__ static constexpr size_t bytes() {
+    return sizeof(double) * 2 * W2 * PairCfg<W2>::BS + (sizeof(double2) + sizeof(double) + sizeof(int2)) * (W2 / 2);
+  }
+};
+
+// P column j (0 <= j < 2w) of pair (I, J) -> working-matrix column.
+template <int W2>
+__device__ __forceinline__ int pcol(int j, int I, int J) {
+  constexpr int W = W2 / 2;
+  return (j < W) ? I * W + j : J * W + (j - W);
+}
+
+// Upper tiles of P^T P for a panel whose 8-col groups start at ptr[c] (already offset by lane:
+// column 8c + lane/4, row lane%4); `rows` multiple of 16; `rstride` = element stride per row.
+template <int W2>
+__device__ __forceinline__ void gram_tiles(const double* const (&ptr)[W2 / 8], int rows, int rstride,
+                                           double (&acc)[PairCfg<W2>::NTU][2]) {
+  constexpr int CG = W2 / 8;
+#pragma unroll
+  for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
+  for (int r0 = 0; r0 < rows; r0 += 16) {
+    double f[4][CG];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+      for (int c = 0; c < CG; ++c) f[u][c] = ptr[c][(size_t)(r0 + 4 * u) * rstride];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      int t = 0;
+#pragma unroll
+      for (int a = 0; a < CG; ++a)
+#pragma unroll
+        for (int b = a; b < CG; ++b) dmma884(acc[t++], f[u][a], f[u][b]);
+    }
+  }
+}
+
+// Write upper tiles (and their mirrors) into a [W2][BS] SMEM buffer; subtract `diag_sub` on the
+// diagonal (1.0 for E = J^T J - I, 0.0 for the Gram).
+template <int W2>
+__device__ __forceinline__ void store_sym(double* buf, const double (&acc)[PairCfg<W2>::NTU][2],
+                                          int lane, double diag_sub) {
+  constexpr int CG = W2 / 8, BS = PairCfg<W2>::BS;
+  int t = 0;
+#pragma unroll
+  for (int a = 0; a < CG; ++a)
+#pragma unroll
+    for (int b = a; b < CG; ++b, ++t)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int row = 8 * a + (lane >> 2), col = 8 * b + 2 * (lane & 3) + e;
+        const double v = acc[t][e] - ((row == col) ? diag_sub : 0.0);
+        buf[row * BS + col] = v;
+        if (a != b) buf[col * BS + row] = v;
+      }
+}
+
+// X (rows x 2w panel of columns colmap(.), leading dim ld) <- X * J', J' given as B fragments
+// jf[kk][nb] = J'[4kk + l%4][8nb + l/4]. In place, 8-row blocks.
+template <int W2>
+__device__ __forceinline__ void apply_rotation(double* base, int ld, int rows, int I, int J, int lane,
+                                               const double (&jf)[W2 / 4][W2 / 8]) {
+  constexpr int CG = W2 / 8, KK = W2 / 4;
+  const double* pa[KK];
+  double* pc[CG][2];
+#pragma unroll
+  for (int kk = 0; kk < KK; ++kk) pa[kk] = base + (size_t)pcol<W2>(4 * kk + (lane & 3), I, J) * ld + (lane >> 2);
+#pragma unroll
+  for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+    for (int e = 0; e < 2; ++e)
+      pc[nb][e] = base + (size_t)pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
+  for (int r0 = 0; r0 < rows; r0 += 16) {
+    double a[2][KK];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int kk = 0; kk < KK; ++kk) a[h][kk] = pa[kk][r0 + 8 * h];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      double acc[CG][2];
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb) acc[nb][0] = acc[nb][1] = 0.0;
+#pragma unroll
+      for (int kk = 0; kk < KK; ++kk)
+#pragma unroll
+        for (int nb = 0; nb < CG; ++nb) dmma884(acc[nb], a[h][kk], jf[kk][nb]);
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) pc[nb][e][r0 + 8 * h] = acc[nb][e];
+    }
+  }
+}
+
+// One inner EVD step r (round-robin over 2w indices): params, two-sided quad update of B, J update.
+template <int W2>
+__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, int r, int lane, double tol,
+                                         const double (&x)[W2], double (&y)[W2]) {
+  using C = PairCfg<W2>;
+  constexpr int BS = C::BS, NPR = C::NPR;
+  double* B = ws.B;
+  bool rot = false;
+  if (lane < NPR) {
+    const int p = rr_content(2 * lane, r, W2), q = rr_content(2 * lane + 1, r, W2);
+    double c, s, t;
+    rot = rot_params(B[p * BS + p], B[q * BS + q], B[p * BS + q], tol, c, s, t);
+    ws.cs[lane] = make_double2(c, s);
+    ws.tt[lane] = rot ? t : 0.0;
+    ws.pq[lane] = make_int2(p, q);
+  }
+  const bool any = __any_sync(0xffffffffu, rot);
+  __syncwarp();
+  if (any) {
+    // Quads (k, l): rows {p_k, q_k} x cols {p_l, q_l}; B' = G^T B G.
+    const int k = lane / C::LPK;
+    const int2 ik = ws.pq[k];
+    const double2 gk = ws.cs[k];
+    const double tk = ws.tt[k];
+#pragma unroll
+    for (int i = 0; i < C::QPL; ++i) {
+      const int l = (lane % C::LPK) * C::QPL + i;
+      if (l == k) {
+        if (tk != 0.0) {  // annihilated pair: closed-form diagonal, exact zero off-diagonal
+          const double bpq = B[ik.x * BS + ik.y];
+          B[ik.x * BS + ik.x] = fma(tk, bpq, B[ik.x * BS + ik.x]);
+          B[ik.y * BS + ik.y] = fma(-tk, bpq, B[ik.y * BS + ik.y]);
+          B[ik.x * BS + ik.y] = 0.0;
+          B[ik.y * BS + ik.x] = 0.0;
+        }
+      } else {
+        const int2 il = ws.pq[l];
+        const double2 gl = ws.cs[l];
+        const double b00 = B[ik.x * BS + il.x], b01 = B[ik.x * BS + il.y];
+        const double b10 = B[ik.y * BS + il.x], b11 = B[ik.y * BS + il.y];
+        // columns (p_l, q_l): B G_l
+        const double c0 = fma(gl.y, b01, gl.x * b00), c1 = fma(-gl.y, b00, gl.x * b01);
+        const double d0 = fma(gl.y, b11, gl.x * b10), d1 = fma(-gl.y, b10, gl.x * b11);
+        // rows (p_k, q_k): G_k^T (B G_l)
+        B[ik.x * BS + il.x] = fma(gk.y, d0, gk.x * c0);
+        B[ik.x * BS + il.y] = fma(gk.y, d1, gk.x * c1);
+        B[ik.y * BS + il.x] = fma(-gk.y, c0, gk.x * d0);
+        B[ik.y * BS + il.y] = fma(-gk.y, c1, gk.x * d1);
+      }
+    }
+  }
+  // J <- J G in slot order; outputs move to their next slots (register rename).
+#pragma unroll
+  for (int k = 0; k < NPR; ++k) {
+    const double2 g = ws.cs[k];
+    const double a = x[2 * k], b = x[2 * k + 1];
+    y[rr_dest(2 * k, W2)] = fma(g.y, b, g.x * a);
+    y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
+  }
+  __syncwarp();
+  return any;
+}
+
+// Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
+// rotated (A and V panels updated); counts inner sweeps into *inner.
+template <int W2>
+__device__ bool process_pair(const WarpSmem<W2>& ws, double* Wm, int ld, int mrows, double* Vm,
+                             int ldv, int vrows, int I, int J, double tol, int inner_cap, int lane,
+                             int* inner) {
+  using C = PairCfg<W2>;
+  constexpr int CG = C::CG, BS = C::BS;
+  // (1) Gram B = P^T P, P = [W_I W_J] (Alg 1 l.5).
+  {
+    const double* ptr[CG];
+#pragma unroll
+    for (int c = 0; c < CG; ++c) ptr[c] = Wm + (size_t)pcol<W2>(8 * c + (lane >> 2), I, J) * ld + (lane & 3);
+    double acc[C::NTU][2];
+    gram_tiles<W2>(ptr, mrows, 1, acc);
+    store_sym<W2>(ws.B, acc, lane, 0.0);
+  }
+  __syncwarp();
+  // (4) off-norm test on the Gram (Z6): skip the pair if every |b_pq| <= tol sqrt(b_pp b_qq).
+  bool need = false;
+  for (int e = lane; e < W2 * W2; e += 32) {
+    const int p = e / W2, q = e % W2;
+    if (p < q) {
+      const double bpp = ws.B[p * BS + p], bqq = ws.B[q * BS + q];
+      need |= (bpp > 0.0 && bqq > 0.0 && fabs(ws.B[p * BS + q]) > tol * (sqrt(bpp) * sqrt(bqq)));
+    }
+  }
+  if (!__any_sync(0xffffffffu, need)) return false;
+  // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, J accumulated in slot order.
+  double ja[W2], jb[W2];
+#pragma unroll
+  for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
+  bool rotated = false;
+  int isw = 0;
+  for (; isw < inner_cap; ++isw) {
+    // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb, slots back in order.
+    bool any = evd_step<W2>(ws, 0, lane, tol, ja, jb);
+    for (int r = 1; r < W2 - 1; r += 2) {
+      any |= evd_step<W2>(ws, r, lane, tol, jb, ja);
+      any |= evd_step<W2>(ws, r + 1, lane, tol, ja, jb);
+    }
+#pragma unroll
+    for (int s = 0; s < W2; ++s) ja[s] = jb[s];
+    rotated |= any;
+    if (!any) break;
+  }
+  *inner += isw + (isw < inner_cap ? 1 : 0);
+  if (!rotated) return false;
+  // Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2.
+  if (lane < W2) {
+#pragma unroll
+    for (int s = 0; s < W2; ++s) ws.S[lane * BS + s] = ja[s];
+  }
+  __syncwarp();
+  {
+    const double* ptr[CG];
+#pragma unroll
+    for (int c = 0; c < CG; ++c) ptr[c] = ws.S + (lane & 3) * BS + 8 * c + (lane >> 2);
+    double acc[C::NTU][2];
+    gram_tiles<W2>(ptr, W2, BS, acc);
+    __syncwarp();
+    store_sym<W2>(ws.B, acc, lane, 1.0);
+  }
+  __syncwarp();
+  double jn[CG][CG][2];
+#pragma unroll
+  for (int i = 0; i < CG; ++i)
+#pragma unroll
+    for (int j = 0; j < CG; ++j) {
+      double acc[2] = {0.0, 0.0};
+#pragma unroll
+      for (int kk = 0; kk < W2 / 4; ++kk)
+        dmma884(acc, ws.S[(8 * i + (lane >> 2)) * BS + 4 * kk + (lane & 3)],
+                ws.B[(4 * kk + (lane & 3)) * BS + 8 * j + (lane >> 2)]);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        jn[i][j][e] = fma(-0.5, acc[e], ws.S[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e]);
+    }
+  __syncwarp();
+#pragma unroll
+  for (int i = 0; i < CG; ++i)
+#pragma unroll
+    for (int j = 0; j < CG; ++j)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) ws.B[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e] = jn[i][j][e];
+  __syncwarp();
+  double jf[W2 / 4][CG];
+#pragma unroll
+  for (int kk = 0; kk < W2 / 4; ++kk)
+#pragma unroll
+    for (int nb = 0; nb < CG; ++nb) jf[kk][nb] = ws.B[(4 * kk + (lane & 3)) * BS + 8 * nb + (lane >> 2)];
+  // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J.
+  apply_rotation<W2>(Wm, ld, mrows, I, J, lane, jf);
+  apply_rotation<W2>(Vm, ldv, vrows, I, J, lane, jf);
+  return true;
+}
+
+}  // namespace
+
+template <int W2, int NW>
+__global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
+                                                             const int* __restrict__ order) {
+  using C = PairCfg<W2>;
+  const MatDesc d = descs[order[blockIdx.x]];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  constexpr int T = NW * 32;
+  const int M = d.M, N = d.N, mp = d.m_pad, np = d.n_pad;
+  double* Wm = d.W;
+  double* Vm = d.Vw;
+
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  WarpSmem<W2> ws;
+  {
+    unsigned char* p = smem_raw + warp * WarpSmem<W2>::bytes();
+    ws.B = reinterpret_cast<double*>(p);
+    ws.S = ws.B + W2 * C::BS;
+    ws.cs = reinterpret_cast<double2*>(ws.S + W2 * C::BS);
+    ws.tt = reinterpret_cast<double*>(ws.cs + W2 / 2);
+    ws.pq = reinterpret_cast<int2*>(ws.tt + W2 / 2);
+  }
+  __shared__ int s_flags[4];
+  __shared__ int s_inner[NW];
+  if (tid < 4) s_flags[tid] = 0;
+  if (tid < NW) s_inner[tid] = 0;
+
+  // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. ----
+  bool bad = false;
+  for (size_t e = tid; e < (size_t)mp * np; e += T) {
+    const int c = (int)(e / mp), r = (int)(e % mp);
+    double v = 0.0;
+    if (r < M && c < N) {
+      v = d.swapped ? d.A[(size_t)r * d.lda + c] : d.A[(size_t)c * d.lda + r];
+      bad |= !isfinite(v);
+    }
+    Wm[e] = v;
+  }
+  for (size_t e = tid; e < (size_t)np * np; e += T) Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
+  __syncthreads();
+  if (bad) atomicOr(&s_flags[2], 1);
+  __syncthreads();
+  const bool nonfinite = s_flags[2] != 0;
+
+  const int nb = np / C::W;  // column blocks (even)
+  int sweep = 0;
+  bool converged = false;
+  int my_inner = 0;
+  if (!nonfinite) {
+    while (sweep < d.max_sweeps) {
+      bool rot_any = false;
+      for (int step = 0; step < nb - 1; ++step) {
+        for (int p = warp; p < nb / 2; p += NW) {
+          const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
+          rot_any |= process_pair<W2>(ws, Wm, mp, mp, Vm, np, np, I, J, d.tol, d.inner_cap, lane, &my_inner);
+        }
+        __syncthreads();
+      }
+      ++sweep;
+      if (rot_any && lane == 0) s_flags[sweep & 1] = 1;
+      __syncthreads();
+      const bool any = s_flags[sweep & 1] != 0;
+      __syncthreads();
+      if (tid == 0) s_flags[sweep & 1] = 0;
+      if (!any) { converged = true; break; }
+    }
+  }
+  if (lane == 0) s_inner[warp] = my_inner;
+  __syncthreads();
+
+  // ---- Finalisation: sigma, rank, sign (Z15), U = W / sigma, un-orientation. ----
+  double* s_sig = reinterpret_cast<double*>(smem_raw);  // reuse warp buffers: [N]
+  double* s_sgn = s_sig + N;                             // [N]
+  int* s_rank = reinterpret_cast<int*>(s_sgn + N);       // [N]
+  for (int j = warp; j < N; j += NW) {
+    const double* col = Wm + (size_t)j * mp;
+    double a = 0.0;
+    for (int r = lane; r < M; r += 32) a = fma(col[r], col[r], a);
+    for (int off = 16; off > 0; off >>= 1) a += __shfl_xor_sync(0xffffffffu, a, off);
+    const double* vc = Vm + (size_t)j * np;
+    double best = 0.0;
+    int bi = 0x7fffffff;
+    for (int i = lane; i < N; i += 32) {
+      const double v = vc[i];
+      if (fabs(v) > fabs(best)) { best = v; bi = i; }
+    }
+    for (int off = 16; off > 0; off >>= 1) {
+      const double ob = __shfl_xor_sync(0xffffffffu, best, off);
+      const int oi = __shfl_xor_sync(0xffffffffu, bi, off);
+      if (fabs(ob) > fabs(best) || (fabs(ob) == fabs(best) && oi < bi)) { best = ob; bi = oi; }
+    }
+    if (lane == 0) {
+      s_sig[j] = nonfinite ? __longlong_as_double(0x7ff8000000000000ULL) : sqrt(a);
+      s_sgn[j] = (best < 0.0) ? -1.0 : 1.0;
+    }
+  }
+  __syncthreads();
+  for (int j = tid; j < N; j += T) {
+    int rk = 0;
+    if (nonfinite) {
+      rk = j;
+    } else {
+      const double sj = s_sig[j];
+      for (int i = 0; i < N; ++i) {
+        const double si = s_sig[i];
+        rk += (si > sj) || (si == sj && i < j);
+      }
+    }
+    s_rank[j] = rk;
+  }
+  __syncthreads();
+  double sig1 = 0.0;
+  for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
+  const double thresh = sig1 * (double)M * kU53;
+  const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
+  double* dstW = d.swapped ? d.V : d.U;
+  const int ldW = d.swapped ? d.ldv : d.ldu;
+  double* dstV = d.swapped ? d.U : d.V;
+  const int ldV = d.swapped ? d.ldu : d.ldv;
+  bool needs_completion = false;
+  for (int j = warp; j < N; j += NW) {
+    const int rk = s_rank[j];
+    const double sj = s_sig[j], sgn = s_sgn[j];
+    const bool ok = sj > thresh;
+    needs_completion |= !ok;
+    if (dstW) {
+      const double* col = Wm + (size_t)j * mp;
+      for (int r = lane; r < M; r += 32)
+        dstW[(size_t)rk * ldW + r] = nonfinite ? nanv : (ok ? sgn * (col[r] / sj) : sgn * 0.0);
+    }
+    if (dstV) {
+      const double* vc = Vm + (size_t)j * np;
+      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = nonfinite ? nanv : sgn * vc[i];
+    }
+    if (lane == 0) d.S[rk] = sj;
+  }
+  if (needs_completion && !nonfinite && lane == 0) atomicOr(&s_flags[3], 1);
+  __syncthreads();
+  if (tid == 0) {
+    int inner = 0;
+    for (int w = 0; w < NW; ++w) inner += s_inner[w];
+    if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
+    if (d.sweeps_inner) d.sweeps_inner[d.idx] = inner;
+    if (d.status) d.status[d.idx] = (s_flags[3] && dstW) ? kNeedsCompletion : 0;
+  }
+}
+
+template <int W2, int NW>
+static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
+  size_t smem = NW * WarpSmem<W2>::bytes();
+  const size_t fin = 3 * 8 * 1024;  // finalisation arrays alias the warp buffers
+  if (smem < fin) smem = fin;
+  auto kern = l1_gram_kernel<W2, NW>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  kern<<<count, NW * 32, smem, stream>>>(descs, order);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
+  switch (variant) {
+    case kL1_16x4: return launch_l1_t<16, 4>(descs, order, count, stream);
+    case kL1_32x4: return launch_l1_t<32, 4>(descs, order, count, stream);
+    case kL1_32x8: return launch_l1_t<32, 8>(descs, order, count, stream);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace wcsvd

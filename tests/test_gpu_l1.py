@@ -1,0 +1,72 @@
+"""Parity of the Level-1 Gram path (Gram -> EVD -> DMMA update -> off-norm test; Alg 1 / Alg 2
+l.10-11) with the oracle, on ragged shapes and the C3/C4 workloads."""
+import numpy as np
+import pytest
+
+import workloads
+import paper_conf_sc_xiaopxsmmlzt22_b200 as wc
+from tests.gpu_helpers import check_parity, gpu_svd_list, gpu_svd_tensor
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("shapes", [
+    [(97, 97), (128, 128), (130, 99), (99, 130), (200, 120)],
+    [(256, 256), (300, 170), (170, 300), (1024, 100), (100, 1024)],
+    [(513, 257), (600, 600)],
+])
+def test_l1_ragged_shapes(shapes):
+    mats = [workloads.gaussian(workloads.matrix_rng(500 + i, 3), m, n) for i, (m, n) in enumerate(shapes)]
+    for (m, n) in shapes:
+        assert wc.plan(m, n)["path"] == wc.PATH_GRAM
+    S, U, V, info = gpu_svd_list(mats)
+    check_parity(mats, S, U, V, info)
+
+
+@pytest.mark.parametrize("w", [8, 16])
+def test_l1_forced_on_small_shapes(w):
+    # The Gram path on shapes the planner would give to Level 0 (ragged tails, m<n, tiny).
+    shapes = [(64, 64), (40, 24), (24, 40), (17, 9), (33, 65), (5, 3)]
+    mats = [workloads.gaussian(workloads.matrix_rng(520 + i, w), m, n) for i, (m, n) in enumerate(shapes)]
+    S, U, V, info = gpu_svd_list(mats, force_path=wc.PATH_GRAM, force_w=w)
+    check_parity(mats, S, U, V, info)
+
+
+def test_l1_ill_conditioned_and_rank_deficient():
+    rng = workloads.matrix_rng(530, 0)
+    mats = []
+    for kappa in (1e6, 1e12):
+        s = kappa ** (-np.arange(150) / 149.0)
+        mats.append(workloads.prescribed(rng, 200, 150, s))
+    Z = workloads.gaussian(rng, 180, 130)
+    Z[:, 5] = 0.0
+    Z[:, 77] = 0.0
+    mats.append(Z)
+    mats.append(workloads.gaussian(rng, 150, 3) @ workloads.gaussian(rng, 3, 140))
+    S, U, V, info = gpu_svd_list(mats)
+    check_parity(mats, S, U, V, info)
+
+
+def test_c3_sampled():
+    cfg = workloads.get_config("C3", batch=256)
+    mats = cfg.matrices()
+    S, U, V, info = gpu_svd_tensor(np.stack(mats))
+    assert np.all(info > 0)
+    check_parity(mats, S, U, V, info, idx=list(range(0, 256, 32)))
+
+
+def test_c4_sampled():
+    cfg = workloads.get_config("C4", batch=64)
+    mats = cfg.matrices()
+    S, U, V, info = gpu_svd_tensor(np.stack(mats))
+    assert np.all(info > 0)
+    check_parity(mats, S, U, V, info, idx=list(range(0, 64, 16)))
+    for k in range(0, 64, 16):
+        assert np.abs(S[k] - cfg.spectrum(k)).max() <= 1e-13
+
+
+def test_l1_bitwise_deterministic_across_batch_composition():
+    mats = [workloads.gaussian(workloads.matrix_rng(540, i), 160, 140) for i in range(6)]
+    S1, U1, V1, _ = gpu_svd_list(mats)
+    S2, U2, V2, _ = gpu_svd_list([mats[3]] + [workloads.gaussian(workloads.matrix_rng(541, 0), 300, 200)])
+    assert np.array_equal(S1[3], S2[0]) and np.array_equal(U1[3], U2[0]) and np.array_equal(V1[3], V2[0])
