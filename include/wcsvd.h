@@ -94,8 +94,9 @@ typedef struct {
   void* workspace;         /* DEVICE buffer or NULL (-> stream-ordered internal allocation) */
   size_t workspace_bytes;  /* size of `workspace`; must be >= wcsvd_workspace_size(...) */
   int force_path;          /* 0 = planner; else WCSVD_PATH_* for every matrix (ablations) */
-  int force_w;             /* 0 = planner; else Level-1 block width w in {8, 16} */
-  int force_w2;            /* 0 = planner; else Level-2 block width (W-cycle path) */
+  int force_w;             /* 0 = planner; else the EVD block width w in {8, 16} (Level 1 of the
+                              Gram path, Level 2 of the W-cycle path) */
+  int wcycle_sweeps;       /* 0 = planner (2); cap on Level-2 sweeps per W-cycle super-pair */
   int inner_sweeps;        /* 0 = planner (1); cap on EVD sweeps per pair */
 } wcsvd_opts;
 

@@ -44,7 +44,7 @@ class OptsT(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_size_t), ("ldu", ctypes.c_void_p), ("ldv", ctypes.c_void_p),
                 ("info", ctypes.c_void_p), ("sweeps_inner", ctypes.c_void_p),
                 ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
-                ("force_path", ctypes.c_int), ("force_w", ctypes.c_int), ("force_w2", ctypes.c_int),
+                ("force_path", ctypes.c_int), ("force_w", ctypes.c_int), ("wcycle_sweeps", ctypes.c_int),
                 ("inner_sweeps", ctypes.c_int)]
 
 
@@ -113,7 +113,7 @@ def _arr_ptr(x) -> np.ndarray:
 def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: float = 0.0,
                     max_sweeps: int = 0, stream: int = 0, ldu=None, ldv=None, info_ptr: int = 0,
                     sweeps_inner_ptr: int = 0, workspace_ptr: int = 0, workspace_bytes: int = 0,
-                    force_path: int = 0, force_w: int = 0, force_w2: int = 0,
+                    force_path: int = 0, force_w: int = 0, wcycle_sweeps: int = 0,
                     inner_sweeps: int = 0) -> None:
     """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError."""
     m, n, lda = _arr_i32(m), _arr_i32(n), _arr_i32(lda)
@@ -132,7 +132,7 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
     opts.sweeps_inner = sweeps_inner_ptr or None
     opts.workspace = workspace_ptr or None
     opts.workspace_bytes = workspace_bytes
-    opts.force_path, opts.force_w, opts.force_w2, opts.inner_sweeps = force_path, force_w, force_w2, inner_sweeps
+    opts.force_path, opts.force_w, opts.wcycle_sweeps, opts.inner_sweeps = force_path, force_w, wcycle_sweeps, inner_sweeps
     rc = lib().wcsvd_batched_ex(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
                                 Sp.ctypes.data, Up.ctypes.data if Up is not None else None,
                                 Vp.ctypes.data if Vp is not None else None, float(tol), int(max_sweeps),

@@ -58,6 +58,16 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   int w = (p->N <= 96) ? 8 : 16;
   if (force_w == 8 || force_w == 16) w = force_w;
   else if (force_w != 0) return WCSVD_ENOTSUP;
+  if (force_path == WCSVD_PATH_WCYCLE) {
+    // Alg 2 l.12-14: w1 = 64 super-blocks recurse to Level 2 with w2 = w (EVD width 2 w2).
+    p->path = WCSVD_PATH_WCYCLE;
+    p->w = 64;
+    p->w2 = w;
+    p->n_pad = (p->N + 127) / 128 * 128;
+    p->m_pad = (p->M + 15) / 16 * 16;
+    p->variant = (w == 8) ? kL1_16x4 : kL1_32x8;
+    return WCSVD_OK;
+  }
   p->path = WCSVD_PATH_GRAM;
   p->w = w;
   p->n_pad = (p->N + 2 * w - 1) / (2 * w) * (2 * w);
@@ -251,6 +261,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     d.tol = (tol > 0) ? tol : std::sqrt((double)p.M) * kU53;
     d.max_sweeps = max_sweeps;
     d.inner_cap = (opts && opts->inner_sweeps > 0) ? opts->inner_sweeps : 1;
+    d.inner_cap2 = (opts && opts->wcycle_sweeps > 0) ? opts->wcycle_sweeps : 2;
     d.idx = b;
     d.status = d_status;
     if (p.path != WCSVD_PATH_L0) {

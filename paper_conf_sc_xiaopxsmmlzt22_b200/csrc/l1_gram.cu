@@ -44,6 +44,10 @@ __device__ __forceinline__ bool rot_params(double alpha, double beta, double gam
   return true;
 }
 
+__device__ __forceinline__ void named_bar(int id, int count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
 template <int W2>
 struct PairCfg {
   static constexpr int W = W2 / 2;          // block width w
@@ -344,8 +348,10 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
   __shared__ int s_flags[4];
   __shared__ int s_inner[NW];
+  __shared__ int s_grp[2 * NW];
   if (tid < 4) s_flags[tid] = 0;
   if (tid < NW) s_inner[tid] = 0;
+  if (tid < 2 * NW) s_grp[tid] = 0;
 
   // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. ----
   bool bad = false;
@@ -364,17 +370,69 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __syncthreads();
   const bool nonfinite = s_flags[2] != 0;
 
-  const int nb = np / C::W;  // column blocks (even)
   int sweep = 0;
   bool converged = false;
   int my_inner = 0;
-  if (!nonfinite) {
+  if (!nonfinite && d.w2 == 0) {
+    // Flat Level 1: round-robin over the n_pad / w column blocks (Alg 1).
+    const int nb = np / C::W;
     while (sweep < d.max_sweeps) {
       bool rot_any = false;
       for (int step = 0; step < nb - 1; ++step) {
         for (int p = warp; p < nb / 2; p += NW) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
           rot_any |= process_pair<W2>(ws, Wm, mp, mp, Vm, np, np, I, J, d.tol, d.inner_cap, lane, &my_inner);
+        }
+        __syncthreads();
+      }
+      ++sweep;
+      if (rot_any && lane == 0) s_flags[sweep & 1] = 1;
+      __syncthreads();
+      const bool any = s_flags[sweep & 1] != 0;
+      __syncthreads();
+      if (tid == 0) s_flags[sweep & 1] = 0;
+      if (!any) { converged = true; break; }
+    }
+  } else if (!nonfinite) {
+    // W-cycle (Alg 2 l.12-14; Step 3; Fig 3-4): Level-1 super-blocks
+    // of width w1 = d.w are paired round-robin; each super-pair panel [A_I A_J] (M x 2 w1) fits no
+    // on-chip EVD, so it recurses to Level 2: block Jacobi with w2 = d.w2 (the EVD width W2/2) over
+    // its 2r sub-blocks (r = w1 / w2) until they are mutually orthogonal or inner_cap2 Level-2
+    // sweeps ran. The Level-2 rotations are applied to the A and V sub-panels as they are found, so
+    // the panel leaves Level 2 already rotated and V carries J_IJ (Z23: no separate A update).
+    // A group of GS warps owns one super-pair; named barriers separate its Level-2 steps.
+    const int r = d.w / C::W;
+    const int nb1 = np / d.w;
+    const int GS = (r < NW) ? r : NW, NG = NW / GS;
+    const int grp = warp / GS, gw = warp % GS;
+    const bool active_grp = grp < NG;
+    while (sweep < d.max_sweeps) {
+      bool rot_any = false;
+      for (int s1 = 0; s1 < nb1 - 1; ++s1) {
+        if (active_grp) {
+          for (int p1 = grp; p1 < nb1 / 2; p1 += NG) {
+            const int I1 = rr_content(2 * p1, s1, nb1), J1 = rr_content(2 * p1 + 1, s1, nb1);
+            for (int isw = 0; isw < d.inner_cap2; ++isw) {
+              bool mine = false;
+              for (int s2 = 0; s2 < 2 * r - 1; ++s2) {
+                for (int p2 = gw; p2 < r; p2 += GS) {
+                  const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
+                  const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
+                  const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
+                  mine |= process_pair<W2>(ws, Wm, mp, mp, Vm, np, np, Ia, Ib, d.tol, d.inner_cap, lane, &my_inner);
+                }
+                named_bar(1 + grp, GS * 32);
+              }
+              // group vote on "some Level-2 pair rotated in this inner sweep"
+              if (mine && lane == 0) s_grp[grp * 2 + (isw & 1)] = 1;
+              named_bar(1 + grp, GS * 32);
+              const bool any2 = s_grp[grp * 2 + (isw & 1)] != 0;
+              named_bar(1 + grp, GS * 32);
+              if (gw == 0 && lane == 0) s_grp[grp * 2 + (isw & 1)] = 0;
+              rot_any |= any2;
+              if (!any2) break;
+            }
+          }
         }
         __syncthreads();
       }

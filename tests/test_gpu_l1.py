@@ -70,3 +70,42 @@ def test_l1_bitwise_deterministic_across_batch_composition():
     S1, U1, V1, _ = gpu_svd_list(mats)
     S2, U2, V2, _ = gpu_svd_list([mats[3]] + [workloads.gaussian(workloads.matrix_rng(541, 0), 300, 200)])
     assert np.array_equal(S1[3], S2[0]) and np.array_equal(U1[3], U2[0]) and np.array_equal(V1[3], V2[0])
+
+
+@pytest.mark.parametrize("w", [8, 16])
+def test_wcycle_forced(w):
+    # W-cycle recursion (Alg 2 l.12-14): Level-1 super-blocks w1 = 64 -> Level-2 EVD width w2 = w.
+    shapes = [(256, 256), (300, 200), (200, 300), (1024, 130), (150, 140), (130, 129)]
+    mats = [workloads.gaussian(workloads.matrix_rng(550 + i, w), m, n) for i, (m, n) in enumerate(shapes)]
+    for (m, n) in shapes:
+        p = wc.plan(m, n, force_path=wc.PATH_WCYCLE, force_w=w)
+        assert p["path"] == wc.PATH_WCYCLE and p["w"] == 64 and p["w2"] == w
+    S, U, V, info = gpu_svd_list(mats, force_path=wc.PATH_WCYCLE, force_w=w)
+    check_parity(mats, S, U, V, info)
+
+
+def test_wcycle_ill_conditioned():
+    rng = workloads.matrix_rng(560, 0)
+    s = 1e10 ** (-np.arange(200) / 199.0)
+    mats = [workloads.prescribed(rng, 260, 200, s)]
+    S, U, V, info = gpu_svd_list(mats, force_path=wc.PATH_WCYCLE)
+    check_parity(mats, S, U, V, info)
+
+
+def test_c5_mixed_sampled_and_1024_properties():
+    # C5 mixed sizes (first 201 matrices incl. k = 0, 100, 200 forced to 1024x1024): oracle parity on
+    # the matrices with min(m, n) <= 160 (seconds in long double), and for the 1024^2 ones the
+    # size-independent properties plus LAPACK sigma.
+    cfg = workloads.get_config("C5", batch=201)
+    mats = cfg.matrices()
+    S, U, V, info = gpu_svd_list(mats)
+    assert np.all(info > 0)
+    small = [k for k, (m, n) in enumerate(cfg.sizes) if min(m, n) <= 160][:12]
+    check_parity(mats, S, U, V, info, idx=small)
+    from oracle import compare
+    for k in (0, 100, 200):
+        A = mats[k]
+        assert compare.residual(A, S[k], U[k], V[k]) <= 1e-12
+        assert compare.orthogonality(U[k]) <= 1e-11 and compare.orthogonality(V[k]) <= 1e-11
+        s_ref = np.linalg.svd(A, compute_uv=False)
+        assert np.abs(S[k] - s_ref).max() / s_ref[0] <= 1e-12
