@@ -224,6 +224,14 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     if (opts->workspace_bytes < ws_bytes) return -12;
     ws = static_cast<unsigned char*>(opts->workspace);
   } else {
+    // Stream-ordered allocation from the device's default pool. Keep freed blocks cached in the
+    // pool (release threshold = max) so repeated calls do not re-map gigabytes of workspace.
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
     if (cudaMallocAsync(reinterpret_cast<void**>(&ws), ws_bytes, stream) != cudaSuccess) {
       cudaGetLastError();
       return WCSVD_ENOMEM;
@@ -281,14 +289,41 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     e = cudaMemcpyAsync(d_order, h_order.data(), sizeof(int) * batch, cudaMemcpyHostToDevice, stream);
 
   // ---- launches ----
-  for (size_t i = 0; i < buckets.size() && e == cudaSuccess; ++i) {
+  // One launch per plan bucket (largest first). With several buckets (mixed sizes) each runs on its
+  // own stream forked from `stream` so small buckets fill the SMs that large ones leave idle; all
+  // are joined back into `stream` before the completion pass. Per-matrix results do not depend on
+  // this concurrency (each CTA owns one matrix).
+  const int nbk = (int)buckets.size();
+  std::vector<cudaStream_t> side(nbk > 1 ? nbk : 0, nullptr);
+  std::vector<cudaEvent_t> done(side.size(), nullptr);
+  cudaEvent_t fork = nullptr;
+  if (nbk > 1 && e == cudaSuccess) {
+    e = cudaEventCreateWithFlags(&fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(fork, stream);
+    for (int i = 0; i < nbk && e == cudaSuccess; ++i) {
+      e = cudaStreamCreateWithFlags(&side[i], cudaStreamNonBlocking);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming);
+      if (e == cudaSuccess) e = cudaStreamWaitEvent(side[i], fork, 0);
+    }
+  }
+  for (int i = 0; i < nbk && e == cudaSuccess; ++i) {
     const Bucket& bk = buckets[i];
     const int cnt = (int)bk.members.size();
+    cudaStream_t st = (nbk > 1) ? side[i] : stream;
     if (bk.path == WCSVD_PATH_L0)
-      e = launch_l0(bk.variant, d_descs, d_order + bucket_off[i], cnt, bk.maxM, stream);
+      e = launch_l0(bk.variant, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
-      e = launch_l1(bk.variant, d_descs, d_order + bucket_off[i], cnt, stream);
+      e = launch_l1(bk.variant, d_descs, d_order + bucket_off[i], cnt, st);
+    if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);
   }
+  for (int i = 0; i < (int)side.size(); ++i) {
+    if (e == cudaSuccess && done[i]) e = cudaStreamWaitEvent(stream, done[i], 0);
+  }
+  for (int i = 0; i < (int)side.size(); ++i) {
+    if (done[i]) cudaEventDestroy(done[i]);
+    if (side[i]) cudaStreamDestroy(side[i]);  // released once its work completes
+  }
+  if (fork) cudaEventDestroy(fork);
   if (e == cudaSuccess) e = launch_complete(d_descs, batch, stream);
   if (own_ws) cudaFreeAsync(ws, stream);
   if (e != cudaSuccess) {

@@ -22,50 +22,30 @@
 
 #include "common.cuh"
 #include "kernels.h"
+#include "rotation.cuh"
 
 namespace wcsvd {
 
 namespace {
 
-// Rotation of eq (4) for squared norms alpha, beta and dot product gamma, with the
-// threshold test of SURVEY Z5/Z6. tau = (alpha - beta)/(2 gamma) and
-// t = sgn(tau)/(|tau| + sqrt(1 + tau^2)) are evaluated as t = sgn(tau) 2|gamma| / (|d| + sqrt(d^2 +
-// 4 gamma^2)), d = alpha - beta (the same number, multiplied through by 2|gamma|; one division
-// instead of three). sgn(0) = +1 (Z4). Valid while d^2 + 4 gamma^2 does not overflow (column norms
-// below ~1e150). Returns true (and c, s, t) if the pair rotates.
-__device__ __forceinline__ bool jacobi_rot(double alpha, double beta, double gamma, double tol,
-                                           double& c, double& s, double& t) {
-  c = 1.0; s = 0.0; t = 0.0;
-  if (alpha == 0.0 || beta == 0.0) return false;
-  if (fabs(gamma) <= tol * (sqrt(alpha) * sqrt(beta))) return false;
-  const double d = alpha - beta;
-  const double r = sqrt(fma(d, d, 4.0 * gamma * gamma));
-  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 1.0 : -1.0;  // sgn(tau)
-  t = sg * (2.0 * fabs(gamma)) / (fabs(d) + r);
-  c = rsqrt(fma(t, t, 1.0));  // c = 1/sqrt(1+t^2)
-  s = t * c;                  // s = t c
-  return true;
-}
-
 // Per-CTA state shared by the step functions.
 struct L0Ctx {
-  double* part_g;  // [RW][PS] partial gamma per (row-thread, pair)
-  double* part_a;  // [RW][PS] partial alpha (first step of a sweep)
-  double* part_b;  // [RW][PS] partial beta
-  double* nrm;     // [2][NP]  cached squared norms per slot, double-buffered by step parity
-  double2* cs;     // [G][LP+1] (c, s) per pair, padded against bank conflicts
-  int* flags;      // [0],[1] rotation flag per sweep parity; [2] non-finite; [3] completion
-  int RW, PS;
-  int tid, g, rt;
+  double* part;    // [2 parity][3][RW4][PS]: partial gamma / alpha / beta per (row-thread, pair)
+  double* nrm;     // this warp's [2][NP] cached squared norms per slot (step parity)
+  double2* cs;     // this warp's [G][LP+1] (c, s) per pair (padded against bank conflicts)
+  int RW4, PS;
+  int lane, g, rt;
   bool isW;
-  int dtop, dbot;  // reducer lane k: slots that the contents of slots 2k, 2k+1 move to
-  double tol;
-  int gs;          // global step counter
-  int sweep;       // completed sweeps
+  int dtop, dbot;  // lane k: the slots that the contents of slots 2k, 2k+1 move to
+  double tol2;
+  int gs;          // global step counter (parity of the partial and norm buffers)
+  bool rot_sweep;  // some rotation in the current sweep (identical in every warp)
 };
 
 // One round-robin step: every pair of the matrix is orthogonalised once; reads the
-// slots from x, writes the rotated, moved slots to y.
+// slots from x, writes the rotated, moved slots to y. One CTA barrier per step: every warp reduces
+// the row-thread partials itself (lane k = pair k, fixed order) and computes the same rotations,
+// so the (c, s) broadcast needs no second barrier; results are bitwise identical across warps.
 template <int NP, int G, int R, bool FIRST>
 __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
                                         double (&y)[R][NP / G]) {
@@ -74,6 +54,9 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
   constexpr int NPAIR = NP / 2;
   static_assert(LP >= 2 && NPAIR <= 32, "L0 tile");
   const int g = cx.g;
+  const int par = cx.gs & 1;
+  const int SEC = cx.RW4 * cx.PS;  // one partial section
+  double* part = cx.part + par * 3 * SEC;
   // Phase 1: this thread's partial dot products for its pairs (and squared norms at sweep start).
   if (cx.isW) {
     const int base = cx.rt * cx.PS + g * LP;
@@ -88,51 +71,50 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
           be = fma(x[r][2 * j + 1], x[r][2 * j + 1], be);
         }
       }
-      cx.part_g[base + j] = gm;
+      part[base + j] = gm;
       if (FIRST) {
-        cx.part_a[base + j] = al;
-        cx.part_b[base + j] = be;
+        part[SEC + base + j] = al;
+        part[2 * SEC + base + j] = be;
       }
     }
   }
   __syncthreads();
-  // Phase 2 (warp 0, lane k = pair k): fixed-order sum over row-threads, eq (4), eq (6).
-  if (cx.tid < 32) {
-    if (FIRST && cx.tid == 0) cx.flags[(cx.sweep + 1) & 1] = 0;
-    const int k = cx.tid;
+  // Phase 2 (every warp; lane k = pair k): fixed-order sum over row-threads, eq (4), eq (6).
+  bool rot = false;
+  {
+    const int k = cx.lane;
     if (k < NPAIR) {
-      const int PS = cx.PS, RW = cx.RW;
+      const int PS = cx.PS;
       double g4[4] = {0.0, 0.0, 0.0, 0.0}, a4[4] = {0.0, 0.0, 0.0, 0.0}, b4[4] = {0.0, 0.0, 0.0, 0.0};
-      // rows [RW, RW4) of the partial arrays are zero (set once at kernel start)
-      for (int i = 0; i < RW; i += 4) {
+      for (int i = 0; i < cx.RW4; i += 4) {  // rows [RW, RW4) are zero
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          g4[u] += cx.part_g[(i + u) * PS + k];
+          g4[u] += part[(i + u) * PS + k];
           if (FIRST) {
-            a4[u] += cx.part_a[(i + u) * PS + k];
-            b4[u] += cx.part_b[(i + u) * PS + k];
+            a4[u] += part[SEC + (i + u) * PS + k];
+            b4[u] += part[2 * SEC + (i + u) * PS + k];
           }
         }
       }
       const double gm = (g4[0] + g4[1]) + (g4[2] + g4[3]);
-      const int cur = cx.gs & 1;
       double al, be;
       if (FIRST) {
         al = (a4[0] + a4[1]) + (a4[2] + a4[3]);
         be = (b4[0] + b4[1]) + (b4[2] + b4[3]);
       } else {
-        al = cx.nrm[cur * NP + 2 * k];
-        be = cx.nrm[cur * NP + 2 * k + 1];
+        al = cx.nrm[par * NP + 2 * k];
+        be = cx.nrm[par * NP + 2 * k + 1];
       }
-      double c, s, t;
-      const bool rot = jacobi_rot(al, be, gm, cx.tol, c, s, t);
-      cx.cs[(k / LP) * (LP + 1) + (k % LP)] = make_double2(c, s);
-      cx.nrm[(cur ^ 1) * NP + cx.dtop] = rot ? fma(t, gm, al) : al;
-      cx.nrm[(cur ^ 1) * NP + cx.dbot] = rot ? fma(-t, gm, be) : be;
-      if (rot) cx.flags[cx.sweep & 1] = 1;
+      double c, sn, t;
+      rot = jacobi_rotation(al, be, gm, cx.tol2, c, sn, t);
+      cx.cs[(k / LP) * (LP + 1) + (k % LP)] = make_double2(c, sn);
+      // eq (6) in closed form: alpha' = alpha + t gamma, beta' = beta - t gamma
+      cx.nrm[(par ^ 1) * NP + cx.dtop] = rot ? fma(t, gm, al) : al;
+      cx.nrm[(par ^ 1) * NP + cx.dbot] = rot ? fma(-t, gm, be) : be;
     }
   }
-  __syncthreads();
+  cx.rot_sweep |= (__ballot_sync(0xffffffffu, rot) != 0u);
+  __syncwarp();
   // Phase 3: rotate this thread's rows of X or V (eq 3) and move the slots (common.cuh ring).
   // Outputs of local pair j: top -> top[j+1], bot -> bot[j-1]. Group 0 keeps top[0] and sends
   // bot[0] to its top[1]; other groups receive top[0] from the left neighbour lane; the last group
@@ -173,6 +155,7 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
 // One sweep of NP-1 steps starting in x; ends in y with every slot back in its original column.
 template <int NP, int G, int R>
 __device__ __forceinline__ void l0_sweep(L0Ctx& cx, double (&x)[R][NP / G], double (&y)[R][NP / G]) {
+  cx.rot_sweep = false;
   l0_step<NP, G, R, true>(cx, x, y);
   for (int i = 0; i < (NP - 2) / 2; ++i) {
     l0_step<NP, G, R, false>(cx, y, x);
@@ -184,13 +167,15 @@ __device__ __forceinline__ void l0_sweep(L0Ctx& cx, double (&x)[R][NP / G], doub
 
 // Shared-memory bytes of one CTA (must match the carve-up in the kernel).
 template <int NP, int G, int R>
-size_t l0_smem_bytes(int M) {
-  const int RW = ((M + R - 1) / R + 3) / 4 * 4;
+size_t l0_smem_bytes(int M, int threads) {
+  const int RW4 = ((M + R - 1) / R + 3) / 4 * 4;
   const int PS = NP / 2 + 1;
   const int RV = NP / R;
   const int LP = NP / G / 2;
-  return sizeof(double2) * G * (LP + 1) + sizeof(double) * (2 * NP + 2 * NP + (size_t)RV * NP) +
-         sizeof(double) * 3 * (size_t)RW * PS + sizeof(int) * (NP + 8);
+  const int NW = threads / 32;
+  return sizeof(double) * 6 * (size_t)RW4 * PS                         // partials, 2 parities
+         + (size_t)NW * (sizeof(double2) * G * (LP + 1) + sizeof(double) * 2 * NP)  // per-warp cs, nrm
+         + sizeof(double) * (2 * NP + (size_t)RV * NP) + sizeof(int) * (NP + 8);
 }
 
 // One CTA per matrix. Thread t: group g = t % G, row-thread rt = t / G. Row-threads [0, RW) hold
@@ -215,22 +200,26 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   const bool isV = !isW && rt < RW + RV;
 
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  double2* s_cs = reinterpret_cast<double2*>(smem_raw);  // [G][LP+1]
-  double* s_nrm = reinterpret_cast<double*>(s_cs + G * (LP + 1));  // [2][NP]
-  double* s_sig = s_nrm + 2 * NP;                        // [NP]
-  double* s_sgn = s_sig + NP;                            // [NP]
-  double* s_vbest = s_sgn + NP;                          // [RV][NP]
-  const int RW4 = (RW + 3) / 4 * 4;                      // partial rows padded to 4 (zeros)
-  double* s_part = s_vbest + RV * NP;                    // [3][RW4][PS]
-  int* s_rank = reinterpret_cast<int*>(s_part + 3 * RW4 * PS);  // [NP]
-  int* s_flags = s_rank + NP;                            // [8]
-  if (tid < 8) s_flags[tid] = 0;
-  for (int e = tid; e < 3 * RW4 * PS; e += T) s_part[e] = 0.0;
+  const int RW4 = (RW + 3) / 4 * 4;  // partial rows padded to 4 (zeros)
+  const int NWARP = T / 32;
+  double* s_part = reinterpret_cast<double*>(smem_raw);                   // [2][3][RW4][PS]
+  double2* s_csw = reinterpret_cast<double2*>(s_part + 6 * RW4 * PS);     // [NWARP][G][LP+1]
+  double* s_nrmw = reinterpret_cast<double*>(s_csw + NWARP * G * (LP + 1));  // [NWARP][2][NP]
+  double* s_sig = s_nrmw + NWARP * 2 * NP;                                // [NP]
+  double* s_sgn = s_sig + NP;                                             // [NP]
+  double* s_vbest = s_sgn + NP;                                           // [RV][NP]
+  int* s_rank = reinterpret_cast<int*>(s_vbest + RV * NP);                // [NP]
+  int* s_flags = s_rank + NP;                                             // [8]
+  unsigned long long* s_max = reinterpret_cast<unsigned long long*>(s_flags + 4);
+  if (tid < 4) s_flags[tid] = 0;
+  if (tid == 0) *s_max = 0ull;
+  for (int e = tid; e < 6 * RW4 * PS; e += T) s_part[e] = 0.0;
   __syncthreads();
 
   // ---- Stage-in: X = A (m >= n) or A^T (m < n), zero-padded; V = I. ----
   double xa[R][NL], xb[R][NL];
   bool bad = false;
+  double amax = 0.0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
 #pragma unroll
@@ -242,6 +231,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
         if (row < M && col < N) {
           v = d.swapped ? d.A[(size_t)row * d.lda + col] : d.A[(size_t)col * d.lda + row];
           bad |= !isfinite(v);
+          amax = fmax(amax, fabs(v));
         }
       } else if (isV) {
         v = ((rt - RW) * R + r == col) ? 1.0 : 0.0;
@@ -250,42 +240,55 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
     }
   }
   if (bad) atomicOr(&s_flags[2], 1);
+  if (isW && amax > 0.0) atomicMax(s_max, (unsigned long long)__double_as_longlong(amax));
   __syncthreads();
   const bool nonfinite = s_flags[2] != 0;
+  // Exact power-of-two pre-scaling to max|x| in [0.5, 1): every product in the iteration stays in
+  // range, and (no under/overflow) the rotations, U and V are bitwise those of the unscaled input
+  // (SURVEY P10); sigma is scaled back at finalisation.
+  int sexp = 0;
+  if (!nonfinite && *s_max != 0ull) {
+    frexp(__longlong_as_double((long long)*s_max), &sexp);
+    if (isW) {
+      const double f = ldexp(1.0, -sexp);
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+#pragma unroll
+        for (int l = 0; l < NL; ++l) xa[r][l] *= f;
+    }
+  }
 
+  const int lane = tid & 31, warp = tid >> 5;
   L0Ctx cx;
-  cx.part_g = s_part;
-  cx.part_a = s_part + RW4 * PS;
-  cx.part_b = s_part + 2 * RW4 * PS;
-  cx.nrm = s_nrm;
-  cx.cs = s_cs;
-  cx.flags = s_flags;
-  cx.RW = RW;
+  cx.part = s_part;
+  cx.nrm = s_nrmw + warp * 2 * NP;
+  cx.cs = s_csw + warp * G * (LP + 1);
+  cx.RW4 = RW4;
   cx.PS = PS;
-  cx.tid = tid;
+  cx.lane = lane;
   cx.g = g;
   cx.rt = rt;
   cx.isW = isW;
-  cx.dtop = rr_dest(2 * (tid % 32), NP);
-  cx.dbot = rr_dest(2 * (tid % 32) + 1, NP);
-  cx.tol = d.tol;
+  cx.dtop = rr_dest(2 * lane, NP);
+  cx.dbot = rr_dest(2 * lane + 1, NP);
+  cx.tol2 = d.tol * d.tol;
   cx.gs = 0;
-  cx.sweep = 0;
+  cx.rot_sweep = false;
+  int sweep = 0;
   bool converged = false;
   bool in_b = false;
   if (!nonfinite) {
     for (;;) {
       l0_sweep<NP, G, R>(cx, xa, xb);  // ends in xb
-      ++cx.sweep;
-      if (s_flags[(cx.sweep - 1) & 1] == 0) { converged = true; in_b = true; break; }
-      if (cx.sweep >= d.max_sweeps) { in_b = true; break; }
+      ++sweep;
+      if (!cx.rot_sweep) { converged = true; in_b = true; break; }
+      if (sweep >= d.max_sweeps) { in_b = true; break; }
       l0_sweep<NP, G, R>(cx, xb, xa);  // ends in xa
-      ++cx.sweep;
-      if (s_flags[(cx.sweep - 1) & 1] == 0) { converged = true; break; }
-      if (cx.sweep >= d.max_sweeps) break;
+      ++sweep;
+      if (!cx.rot_sweep) { converged = true; break; }
+      if (sweep >= d.max_sweeps) break;
     }
   }
-  const int sweep = cx.sweep;
   if (in_b) {
 #pragma unroll
     for (int r = 0; r < R; ++r)
@@ -324,7 +327,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
 #pragma unroll
       for (int u = 0; u < 4; ++u) a4[u] += s_part[base + (i + u) * PS];
     }
-    s_sig[j] = sqrt((a4[0] + a4[1]) + (a4[2] + a4[3]));
+    s_sig[j] = sqrt((a4[0] + a4[1]) + (a4[2] + a4[3]));  // of the pre-scaled X
     double best = 0.0;
     for (int i = 0; i < RV; ++i) {
       const double v = s_vbest[i * NP + j];
@@ -350,7 +353,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   __syncthreads();
   double sig1 = 0.0;
   for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
-  const double thresh = sig1 * (double)M * kU53;  // Z14 rank threshold
+  const double thresh = sig1 * (double)M * kU53;  // Z14 rank threshold (scale-invariant)
   const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
   // X-space factors: U_w -> U (V if swapped), V_x -> V (U if swapped).
   double* dstW = d.swapped ? d.V : d.U;
@@ -393,7 +396,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
     }
   }
   if (needs_completion && !nonfinite) atomicOr(&s_flags[3], 1);
-  for (int j = tid; j < N; j += T) d.S[s_rank[j]] = nonfinite ? nanv : s_sig[j];
+  for (int j = tid; j < N; j += T) d.S[s_rank[j]] = nonfinite ? nanv : ldexp(s_sig[j], sexp);
   __syncthreads();
   if (tid == 0) {
     if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
@@ -410,7 +413,7 @@ static cudaError_t launch_l0_t(const MatDesc* descs, const int* order, int count
   int threads = (RW + NP / R) * G;
   threads = (threads + 31) / 32 * 32;
   if (threads > MAXT) return cudaErrorInvalidConfiguration;
-  const size_t smem = l0_smem_bytes<NP, G, R>(maxM);
+  const size_t smem = l0_smem_bytes<NP, G, R>(maxM, threads);
   auto kern = l0_jacobi_kernel<NP, G, R, MAXT>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;

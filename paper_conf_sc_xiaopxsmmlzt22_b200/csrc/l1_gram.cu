@@ -24,25 +24,11 @@
 #include "common.cuh"
 #include "dmma.cuh"
 #include "kernels.h"
+#include "rotation.cuh"
 
 namespace wcsvd {
 
 namespace {
-
-__device__ __forceinline__ bool rot_params(double alpha, double beta, double gamma, double tol,
-                                           double& c, double& s, double& t) {
-  // eq (4) / §II.D rho with the threshold of SURVEY Z5/Z6; see l0_jacobi.cu.
-  c = 1.0; s = 0.0; t = 0.0;
-  if (alpha <= 0.0 || beta <= 0.0) return false;
-  if (fabs(gamma) <= tol * (sqrt(alpha) * sqrt(beta))) return false;
-  const double d = alpha - beta;
-  const double r = sqrt(fma(d, d, 4.0 * gamma * gamma));
-  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 1.0 : -1.0;
-  t = sg * (2.0 * fabs(gamma)) / (fabs(d) + r);
-  c = rsqrt(fma(t, t, 1.0));
-  s = t * c;
-  return true;
-}
 
 __device__ __forceinline__ void named_bar(int id, int count) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
@@ -55,8 +41,8 @@ struct PairCfg {
   static constexpr int NTU = CG * (CG + 1) / 2;  // upper tiles of the 2w x 2w Gram
   static constexpr int BS = W2 + 1;         // SMEM row stride of 2w x 2w buffers (doubles)
   static constexpr int NPR = W2 / 2;        // rotation pairs per EVD step
-  static constexpr int LPK = 32 / NPR;      // lanes per row-pair k in the quad phase
-  static constexpr int QPL = NPR / LPK;     // quads per lane
+  static constexpr int NQ = NPR * (NPR - 1) / 2;  // off-diagonal quads (k < l) per EVD step
+  static constexpr int QPL = (NQ + 31) / 32;       // quads per lane
   static_assert(W2 == 16 || W2 == 32, "pair panel width");
 };
 
@@ -83,25 +69,45 @@ __device__ __forceinline__ int pcol(int j, int I, int J) {
 // Upper tiles of P^T P for a panel whose 8-col groups start at ptr[c] (already offset by lane:
 // column 8c + lane/4, row lane%4); `rows` multiple of 16; `rstride` = element stride per row.
 template <int W2>
+__device__ __forceinline__ void gram_load(double (&f)[4][W2 / 8], const double* const (&ptr)[W2 / 8], int r0,
+                                          int rstride) {
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int c = 0; c < W2 / 8; ++c) f[u][c] = ptr[c][(size_t)(r0 + 4 * u) * rstride];
+}
+
+template <int W2>
+__device__ __forceinline__ void gram_mma(double (&acc)[PairCfg<W2>::NTU][2], const double (&f)[4][W2 / 8]) {
+  constexpr int CG = W2 / 8;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    int t = 0;
+#pragma unroll
+    for (int a = 0; a < CG; ++a)
+#pragma unroll
+      for (int b = a; b < CG; ++b) dmma884(acc[t++], f[u][a], f[u][b]);
+  }
+}
+
+// Upper tiles of P^T P for a panel whose 8-col groups start at ptr[c] (already offset by lane:
+// column 8c + lane/4, row lane%4); `rows` multiple of 16; `rstride` = element stride per row.
+// The next 16-row slab is loaded while the current one feeds the DMMAs (register ping-pong).
+template <int W2>
 __device__ __forceinline__ void gram_tiles(const double* const (&ptr)[W2 / 8], int rows, int rstride,
                                            double (&acc)[PairCfg<W2>::NTU][2]) {
   constexpr int CG = W2 / 8;
 #pragma unroll
   for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
-  for (int r0 = 0; r0 < rows; r0 += 16) {
-    double f[4][CG];
-#pragma unroll
-    for (int u = 0; u < 4; ++u)
-#pragma unroll
-      for (int c = 0; c < CG; ++c) f[u][c] = ptr[c][(size_t)(r0 + 4 * u) * rstride];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      int t = 0;
-#pragma unroll
-      for (int a = 0; a < CG; ++a)
-#pragma unroll
-        for (int b = a; b < CG; ++b) dmma884(acc[t++], f[u][a], f[u][b]);
-    }
+  double f0[4][CG], f1[4][CG];
+  gram_load<W2>(f0, ptr, 0, rstride);
+  for (int r0 = 0;;) {
+    if (r0 + 16 < rows) gram_load<W2>(f1, ptr, r0 + 16, rstride);
+    gram_mma<W2>(acc, f0);
+    if ((r0 += 16) >= rows) break;
+    if (r0 + 16 < rows) gram_load<W2>(f0, ptr, r0 + 16, rstride);
+    gram_mma<W2>(acc, f1);
+    if ((r0 += 16) >= rows) break;
   }
 }
 
@@ -125,92 +131,126 @@ __device__ __forceinline__ void store_sym(double* buf, const double (&acc)[PairC
       }
 }
 
-// X (rows x 2w panel of columns colmap(.), leading dim ld) <- X * J', J' given as B fragments
-// jf[kk][nb] = J'[4kk + l%4][8nb + l/4]. In place, 8-row blocks.
+// X (rows x 2w panel of columns pcol(.), leading dim ld) <- X * J', J' given as B fragments
+// jf[kk][nb] = J'[4kk + l%4][8nb + l/4]. In place, 16-row slabs; the next slab's A fragments are
+// loaded while the current slab is multiplied (register ping-pong).
+template <int W2>
+__device__ __forceinline__ void rot_load(double (&a)[2][W2 / 4], const double* base, const int (&oa)[W2 / 4],
+                                         int r0) {
+#pragma unroll
+  for (int h = 0; h < 2; ++h)
+#pragma unroll
+    for (int kk = 0; kk < W2 / 4; ++kk) a[h][kk] = base[oa[kk] + r0 + 8 * h];
+}
+
+template <int W2>
+__device__ __forceinline__ void rot_mma_store(const double (&a)[2][W2 / 4], const double (&jf)[W2 / 4][W2 / 8],
+                                              double* base, const int (&oc)[W2 / 8][2], int r0) {
+  constexpr int CG = W2 / 8, KK = W2 / 4;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    double acc[CG][2];
+#pragma unroll
+    for (int nb = 0; nb < CG; ++nb) acc[nb][0] = acc[nb][1] = 0.0;
+#pragma unroll
+    for (int kk = 0; kk < KK; ++kk)
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb) dmma884(acc[nb], a[h][kk], jf[kk][nb]);
+#pragma unroll
+    for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) base[oc[nb][e] + r0 + 8 * h] = acc[nb][e];
+  }
+}
+
 template <int W2>
 __device__ __forceinline__ void apply_rotation(double* base, int ld, int rows, int I, int J, int lane,
                                                const double (&jf)[W2 / 4][W2 / 8]) {
   constexpr int CG = W2 / 8, KK = W2 / 4;
-  const double* pa[KK];
-  double* pc[CG][2];
+  int oa[KK], oc[CG][2];  // element offsets (a panel is < 2^31 elements)
 #pragma unroll
-  for (int kk = 0; kk < KK; ++kk) pa[kk] = base + (size_t)pcol<W2>(4 * kk + (lane & 3), I, J) * ld + (lane >> 2);
+  for (int kk = 0; kk < KK; ++kk) oa[kk] = pcol<W2>(4 * kk + (lane & 3), I, J) * ld + (lane >> 2);
 #pragma unroll
   for (int nb = 0; nb < CG; ++nb)
 #pragma unroll
-    for (int e = 0; e < 2; ++e)
-      pc[nb][e] = base + (size_t)pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
-  for (int r0 = 0; r0 < rows; r0 += 16) {
-    double a[2][KK];
-#pragma unroll
-    for (int h = 0; h < 2; ++h)
-#pragma unroll
-      for (int kk = 0; kk < KK; ++kk) a[h][kk] = pa[kk][r0 + 8 * h];
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      double acc[CG][2];
-#pragma unroll
-      for (int nb = 0; nb < CG; ++nb) acc[nb][0] = acc[nb][1] = 0.0;
-#pragma unroll
-      for (int kk = 0; kk < KK; ++kk)
-#pragma unroll
-        for (int nb = 0; nb < CG; ++nb) dmma884(acc[nb], a[h][kk], jf[kk][nb]);
-#pragma unroll
-      for (int nb = 0; nb < CG; ++nb)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) pc[nb][e][r0 + 8 * h] = acc[nb][e];
-    }
+    for (int e = 0; e < 2; ++e) oc[nb][e] = pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
+  double a0[2][KK], a1[2][KK];
+  rot_load<W2>(a0, base, oa, 0);
+  for (int r0 = 0;;) {
+    if (r0 + 16 < rows) rot_load<W2>(a1, base, oa, r0 + 16);
+    rot_mma_store<W2>(a0, jf, base, oc, r0);
+    if ((r0 += 16) >= rows) break;
+    if (r0 + 16 < rows) rot_load<W2>(a0, base, oa, r0 + 16);
+    rot_mma_store<W2>(a1, jf, base, oc, r0);
+    if ((r0 += 16) >= rows) break;
   }
 }
 
-// One inner EVD step r (round-robin over 2w indices): params, two-sided quad update of B, J update.
+// Off-diagonal quads (k < l) of an EVD step handled by this lane: q = lane + 32 i.
 template <int W2>
-__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, int r, int lane, double tol,
-                                         const double (&x)[W2], double (&y)[W2]) {
+struct QuadMap {
+  int k[PairCfg<W2>::QPL], l[PairCfg<W2>::QPL];
+  __device__ __forceinline__ void init(int lane) {
+    constexpr int NPR = PairCfg<W2>::NPR, NQ = PairCfg<W2>::NQ;
+#pragma unroll
+    for (int i = 0; i < PairCfg<W2>::QPL; ++i) {
+      int q = lane + 32 * i, kk = 0;
+      k[i] = -1;
+      l[i] = -1;
+      if (q < NQ) {
+        while (q >= NPR - 1 - kk) { q -= NPR - 1 - kk; ++kk; }
+        k[i] = kk;
+        l[i] = kk + 1 + q;
+      }
+    }
+  }
+};
+
+// One inner EVD step r (round-robin over 2w indices): lanes k < w compute the
+// rotations of the step's disjoint pairs (p_k, q_k) and apply the annihilating 2x2 update to their
+// own diagonal quad; then every off-diagonal quad (k < l) of B' = G^T B G is updated from 4 loads
+// and written with its mirror (B symmetric); J <- J G in slot order.
+template <int W2>
+__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, int r, int lane,
+                                         double tol2, const double (&x)[W2], double (&y)[W2]) {
   using C = PairCfg<W2>;
   constexpr int BS = C::BS, NPR = C::NPR;
   double* B = ws.B;
   bool rot = false;
   if (lane < NPR) {
     const int p = rr_content(2 * lane, r, W2), q = rr_content(2 * lane + 1, r, W2);
+    const double bpp = B[p * BS + p], bqq = B[q * BS + q], bpq = B[p * BS + q];
     double c, s, t;
-    rot = rot_params(B[p * BS + p], B[q * BS + q], B[p * BS + q], tol, c, s, t);
+    rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
     ws.cs[lane] = make_double2(c, s);
-    ws.tt[lane] = rot ? t : 0.0;
     ws.pq[lane] = make_int2(p, q);
+    if (rot) {  // annihilated pair: closed-form diagonal (eq 6 analogue), exact zero off-diagonal
+      B[p * BS + p] = fma(t, bpq, bpp);
+      B[q * BS + q] = fma(-t, bpq, bqq);
+      B[p * BS + q] = 0.0;
+      B[q * BS + p] = 0.0;
+    }
   }
   const bool any = __any_sync(0xffffffffu, rot);
   __syncwarp();
   if (any) {
-    // Quads (k, l): rows {p_k, q_k} x cols {p_l, q_l}; B' = G^T B G.
-    const int k = lane / C::LPK;
-    const int2 ik = ws.pq[k];
-    const double2 gk = ws.cs[k];
-    const double tk = ws.tt[k];
 #pragma unroll
     for (int i = 0; i < C::QPL; ++i) {
-      const int l = (lane % C::LPK) * C::QPL + i;
-      if (l == k) {
-        if (tk != 0.0) {  // annihilated pair: closed-form diagonal, exact zero off-diagonal
-          const double bpq = B[ik.x * BS + ik.y];
-          B[ik.x * BS + ik.x] = fma(tk, bpq, B[ik.x * BS + ik.x]);
-          B[ik.y * BS + ik.y] = fma(-tk, bpq, B[ik.y * BS + ik.y]);
-          B[ik.x * BS + ik.y] = 0.0;
-          B[ik.y * BS + ik.x] = 0.0;
-        }
-      } else {
-        const int2 il = ws.pq[l];
-        const double2 gl = ws.cs[l];
+      if (qm.k[i] >= 0) {
+        const int2 ik = ws.pq[qm.k[i]], il = ws.pq[qm.l[i]];
+        const double2 gk = ws.cs[qm.k[i]], gl = ws.cs[qm.l[i]];
         const double b00 = B[ik.x * BS + il.x], b01 = B[ik.x * BS + il.y];
         const double b10 = B[ik.y * BS + il.x], b11 = B[ik.y * BS + il.y];
         // columns (p_l, q_l): B G_l
         const double c0 = fma(gl.y, b01, gl.x * b00), c1 = fma(-gl.y, b00, gl.x * b01);
         const double d0 = fma(gl.y, b11, gl.x * b10), d1 = fma(-gl.y, b10, gl.x * b11);
         // rows (p_k, q_k): G_k^T (B G_l)
-        B[ik.x * BS + il.x] = fma(gk.y, d0, gk.x * c0);
-        B[ik.x * BS + il.y] = fma(gk.y, d1, gk.x * c1);
-        B[ik.y * BS + il.x] = fma(-gk.y, c0, gk.x * d0);
-        B[ik.y * BS + il.y] = fma(-gk.y, c1, gk.x * d1);
+        const double e00 = fma(gk.y, d0, gk.x * c0), e01 = fma(gk.y, d1, gk.x * c1);
+        const double e10 = fma(-gk.y, c0, gk.x * d0), e11 = fma(-gk.y, c1, gk.x * d1);
+        B[ik.x * BS + il.x] = e00; B[il.x * BS + ik.x] = e00;
+        B[ik.x * BS + il.y] = e01; B[il.y * BS + ik.x] = e01;
+        B[ik.y * BS + il.x] = e10; B[il.x * BS + ik.y] = e10;
+        B[ik.y * BS + il.y] = e11; B[il.y * BS + ik.y] = e11;
       }
     }
   }
@@ -229,9 +269,9 @@ __device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, int r, int lane
 // Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
 // rotated (A and V panels updated); counts inner sweeps into *inner.
 template <int W2>
-__device__ bool process_pair(const WarpSmem<W2>& ws, double* Wm, int ld, int mrows, double* Vm,
-                             int ldv, int vrows, int I, int J, double tol, int inner_cap, int lane,
-                             int* inner) {
+__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, double* Wm, int ld, int mrows,
+                             double* Vm, int ldv, int vrows, int I, int J, double tol2, int inner_cap,
+                             int lane, int* inner) {
   using C = PairCfg<W2>;
   constexpr int CG = C::CG, BS = C::BS;
   // (1) Gram B = P^T P, P = [W_I W_J] (Alg 1 l.5).
@@ -244,13 +284,16 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, double* Wm, int ld, int mro
     store_sym<W2>(ws.B, acc, lane, 0.0);
   }
   __syncwarp();
-  // (4) off-norm test on the Gram (Z6): skip the pair if every |b_pq| <= tol sqrt(b_pp b_qq).
+  // (4) off-norm test on the Gram (Z6): skip the pair if every b_pq^2 <= tol^2 b_pp b_qq.
   bool need = false;
-  for (int e = lane; e < W2 * W2; e += 32) {
-    const int p = e / W2, q = e % W2;
-    if (p < q) {
-      const double bpp = ws.B[p * BS + p], bqq = ws.B[q * BS + q];
-      need |= (bpp > 0.0 && bqq > 0.0 && fabs(ws.B[p * BS + q]) > tol * (sqrt(bpp) * sqrt(bqq)));
+  {
+    const double bqq = (lane < W2) ? ws.B[lane * BS + lane] : 0.0;
+#pragma unroll 4
+    for (int p = 0; p < W2 - 1; ++p) {
+      const double bpp = ws.B[p * BS + p];  // broadcast
+      const double bpq = (lane < W2) ? ws.B[p * BS + lane] : 0.0;
+      const double ab = bpp * bqq;
+      need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
     }
   }
   if (!__any_sync(0xffffffffu, need)) return false;
@@ -262,10 +305,10 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, double* Wm, int ld, int mro
   int isw = 0;
   for (; isw < inner_cap; ++isw) {
     // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb, slots back in order.
-    bool any = evd_step<W2>(ws, 0, lane, tol, ja, jb);
+    bool any = evd_step<W2>(ws, qm, 0, lane, tol2, ja, jb);
     for (int r = 1; r < W2 - 1; r += 2) {
-      any |= evd_step<W2>(ws, r, lane, tol, jb, ja);
-      any |= evd_step<W2>(ws, r + 1, lane, tol, ja, jb);
+      any |= evd_step<W2>(ws, qm, r, lane, tol2, jb, ja);
+      any |= evd_step<W2>(ws, qm, r + 1, lane, tol2, ja, jb);
     }
 #pragma unroll
     for (int s = 0; s < W2; ++s) ja[s] = jb[s];
@@ -354,21 +397,37 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   if (tid < 2 * NW) s_grp[tid] = 0;
 
   // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. ----
+  __shared__ unsigned long long s_max;
+  if (tid == 0) s_max = 0ull;
+  __syncthreads();
   bool bad = false;
+  double amax = 0.0;
   for (size_t e = tid; e < (size_t)mp * np; e += T) {
     const int c = (int)(e / mp), r = (int)(e % mp);
     double v = 0.0;
     if (r < M && c < N) {
       v = d.swapped ? d.A[(size_t)r * d.lda + c] : d.A[(size_t)c * d.lda + r];
       bad |= !isfinite(v);
+      amax = fmax(amax, fabs(v));
     }
     Wm[e] = v;
   }
   for (size_t e = tid; e < (size_t)np * np; e += T) Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
-  __syncthreads();
   if (bad) atomicOr(&s_flags[2], 1);
+  if (amax > 0.0) atomicMax(&s_max, (unsigned long long)__double_as_longlong(amax));
   __syncthreads();
   const bool nonfinite = s_flags[2] != 0;
+  // Exact power-of-two pre-scaling to max|w| in [0.5, 1) (see l0_jacobi.cu).
+  int sexp = 0;
+  if (!nonfinite && s_max != 0ull) {
+    frexp(__longlong_as_double((long long)s_max), &sexp);
+    const double f = ldexp(1.0, -sexp);
+    for (size_t e = tid; e < (size_t)mp * np; e += T) Wm[e] *= f;
+  }
+  __syncthreads();
+  const double tol2 = d.tol * d.tol;
+  QuadMap<W2> qm;
+  qm.init(lane);
 
   int sweep = 0;
   bool converged = false;
@@ -381,7 +440,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
       for (int step = 0; step < nb - 1; ++step) {
         for (int p = warp; p < nb / 2; p += NW) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
-          rot_any |= process_pair<W2>(ws, Wm, mp, mp, Vm, np, np, I, J, d.tol, d.inner_cap, lane, &my_inner);
+          rot_any |= process_pair<W2>(ws, qm, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
         }
         __syncthreads();
       }
@@ -419,7 +478,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
-                  mine |= process_pair<W2>(ws, Wm, mp, mp, Vm, np, np, Ia, Ib, d.tol, d.inner_cap, lane, &my_inner);
+                  mine |= process_pair<W2>(ws, qm, Wm, mp, mp, Vm, np, np, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
                 }
                 named_bar(1 + grp, GS * 32);
               }
@@ -512,7 +571,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
       const double* vc = Vm + (size_t)j * np;
       for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = nonfinite ? nanv : sgn * vc[i];
     }
-    if (lane == 0) d.S[rk] = sj;
+    if (lane == 0) d.S[rk] = nonfinite ? sj : ldexp(sj, sexp);
   }
   if (needs_completion && !nonfinite && lane == 0) atomicOr(&s_flags[3], 1);
   __syncthreads();
