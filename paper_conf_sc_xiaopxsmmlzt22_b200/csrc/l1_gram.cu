@@ -25,10 +25,26 @@
 #include "dmma.cuh"
 #include "kernels.h"
 #include "rotation.cuh"
+#include "wcsvd.h"
 
 namespace wcsvd {
 
 namespace {
+
+#ifdef WCSVD_PHASE_PROFILE
+// Debug builds only (-DWCSVD_PHASE_PROFILE): per-phase clock64() totals, lane 0 of every warp.
+__device__ unsigned long long g_phase_cycles[8];
+#define PHASE_T0() long long _pt = clock64()
+#define PHASE_MARK(i)                                                        \
+  do {                                                                       \
+    long long _pn = clock64();                                               \
+    if ((threadIdx.x & 31) == 0) atomicAdd(&g_phase_cycles[i], (unsigned long long)(_pn - _pt)); \
+    _pt = _pn;                                                               \
+  } while (0)
+#else
+#define PHASE_T0() (void)0
+#define PHASE_MARK(i) (void)0
+#endif
 
 __device__ __forceinline__ void named_bar(int id, int count) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
@@ -54,8 +70,15 @@ struct WarpSmem {
   double2* cs;  // [NPR]    (c, s) of the step's rotations
   double* tt;   // [NPR]    t of the step's rotations (0 = none)
   int2* pq;     // [NPR]    (p, q) original indices of the step's pairs
+  double* ring;  // [NSTAGE][W2][SL] cp.async slab ring for the Gram / update panels (aliases B, S)
+  static constexpr int SL = 20;      // ring column stride (doubles): 16 rows + 4 pad (conflict-free fragments)
+  static constexpr int NSTAGE = 3;   // slabs in flight
+  static constexpr int SLAB = W2 * SL;  // doubles per slab
+  __host__ __device__ static constexpr size_t region() {
+    return (2 * W2 * PairCfg<W2>::BS > NSTAGE * SLAB ? 2 * W2 * PairCfg<W2>::BS : NSTAGE * SLAB) * sizeof(double);
+  }
   __host__ __device__ static constexpr size_t bytes() {
-    return sizeof(double) * 2 * W2 * PairCfg<W2>::BS + (sizeof(double2) + sizeof(double) + sizeof(int2)) * (W2 / 2);
+    return region() + (sizeof(double2) + sizeof(double) + sizeof(int2)) * (W2 / 2);
   }
 };
 
@@ -108,6 +131,116 @@ __device__ __forceinline__ void gram_tiles(const double* const (&ptr)[W2 / 8], i
     if (r0 + 16 < rows) gram_load<W2>(f0, ptr, r0 + 16, rstride);
     gram_mma<W2>(acc, f1);
     if ((r0 += 16) >= rows) break;
+  }
+}
+
+// ---- cp.async slab pipeline (per warp): 16-row x 2w-column panel slabs, global -> SMEM ring ----
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// Issue the copy of rows [r0, r0+16) of the 2w panel columns (offsets col_off[c] = pcol(c) * ld) into
+// ring stage `st`: W2 x 8 chunks of 16 B, W2/4 per lane.
+template <int W2>
+__device__ __forceinline__ void slab_issue(const WarpSmem<W2>& ws, const double* base, const int (&coff)[W2 / 4],
+                                           int r0, int st, int lane) {
+  constexpr int SL = WarpSmem<W2>::SL;
+  double* dst = ws.ring + st * WarpSmem<W2>::SLAB;
+#pragma unroll
+  for (int i = 0; i < W2 / 4; ++i) {
+    const int q = lane + 32 * i, c = q >> 3, h = q & 7;
+    cp_async16(dst + c * SL + 2 * h, base + coff[i] + r0 + 2 * h);
+  }
+}
+
+// Column offsets (pcol(c) * ld) of the chunks this lane copies.
+template <int W2>
+__device__ __forceinline__ void slab_offsets(int (&coff)[W2 / 4], int I, int J, int ld, int lane) {
+#pragma unroll
+  for (int i = 0; i < W2 / 4; ++i) coff[i] = pcol<W2>((lane + 32 * i) >> 3, I, J) * ld;
+}
+
+// Upper tiles of P^T P for the global panel of pair (I, J): slabs stream through the ring while
+// the DMMAs consume the previous ones (no register staging, NSTAGE-1 slabs in flight).
+template <int W2>
+__device__ __forceinline__ void gram_tiles_async(const WarpSmem<W2>& ws, const double* base, int ld, int rows,
+                                                 int I, int J, int lane, double (&acc)[PairCfg<W2>::NTU][2]) {
+  constexpr int CG = W2 / 8, SL = WarpSmem<W2>::SL, NS = WarpSmem<W2>::NSTAGE;
+#pragma unroll
+  for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
+  int coff[W2 / 4];
+  slab_offsets<W2>(coff, I, J, ld, lane);
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) slab_issue<W2>(ws, base, coff, 16 * j, j, lane);
+    cp_async_commit();
+  }
+  const int fo = (lane >> 2) * SL + (lane & 3);  // fragment offset inside a column group
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ws, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const double* st = ws.ring + (sl % NS) * WarpSmem<W2>::SLAB;
+    double f[4][CG];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+      for (int c = 0; c < CG; ++c) f[u][c] = st[8 * c * SL + fo + 4 * u];
+    gram_mma<W2>(acc, f);
+    __syncwarp();
+  }
+}
+
+// X <- X * J' for the global panel of pair (I, J), slabs streamed through the ring; results are
+// stored straight to global memory (rows of a slab are read before they are overwritten).
+template <int W2>
+__device__ __forceinline__ void apply_rotation_async(const WarpSmem<W2>& ws, double* base, int ld, int rows,
+                                                     int I, int J, int lane, const double (&jf)[W2 / 4][W2 / 8]) {
+  constexpr int CG = W2 / 8, KK = W2 / 4, SL = WarpSmem<W2>::SL, NS = WarpSmem<W2>::NSTAGE;
+  int coff[W2 / 4];
+  slab_offsets<W2>(coff, I, J, ld, lane);
+  int oc[CG][2];
+#pragma unroll
+  for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) oc[nb][e] = pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) slab_issue<W2>(ws, base, coff, 16 * j, j, lane);
+    cp_async_commit();
+  }
+  const int fo = (lane & 3) * SL + (lane >> 2);  // A fragment: row l/4, column l%4
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ws, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const double* st = ws.ring + (sl % NS) * WarpSmem<W2>::SLAB;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      double a[KK];
+#pragma unroll
+      for (int kk = 0; kk < KK; ++kk) a[kk] = st[4 * kk * SL + fo + 8 * h];
+      double acc[CG][2];
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb) acc[nb][0] = acc[nb][1] = 0.0;
+#pragma unroll
+      for (int kk = 0; kk < KK; ++kk)
+#pragma unroll
+        for (int nb = 0; nb < CG; ++nb) dmma884(acc[nb], a[kk], jf[kk][nb]);
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) __stcg(base + oc[nb][e] + 16 * sl + 8 * h, acc[nb][e]);
+    }
+    __syncwarp();
   }
 }
 
@@ -274,16 +407,15 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, doub
                              int lane, int* inner) {
   using C = PairCfg<W2>;
   constexpr int CG = C::CG, BS = C::BS;
+  PHASE_T0();
   // (1) Gram B = P^T P, P = [W_I W_J] (Alg 1 l.5).
   {
-    const double* ptr[CG];
-#pragma unroll
-    for (int c = 0; c < CG; ++c) ptr[c] = Wm + (size_t)pcol<W2>(8 * c + (lane >> 2), I, J) * ld + (lane & 3);
     double acc[C::NTU][2];
-    gram_tiles<W2>(ptr, mrows, 1, acc);
+    gram_tiles_async<W2>(ws, Wm, ld, mrows, I, J, lane, acc);
     store_sym<W2>(ws.B, acc, lane, 0.0);
   }
   __syncwarp();
+  PHASE_MARK(0);
   // (4) off-norm test on the Gram (Z6): skip the pair if every b_pq^2 <= tol^2 b_pp b_qq.
   bool need = false;
   {
@@ -296,6 +428,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, doub
       need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
     }
   }
+  PHASE_MARK(1);
   if (!__any_sync(0xffffffffu, need)) return false;
   // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, J accumulated in slot order.
   double ja[W2], jb[W2];
@@ -316,6 +449,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, doub
     if (!any) break;
   }
   *inner += isw + (isw < inner_cap ? 1 : 0);
+  PHASE_MARK(2);
   if (!rotated) return false;
   // Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2.
   if (lane < W2) {
@@ -360,9 +494,13 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, doub
   for (int kk = 0; kk < W2 / 4; ++kk)
 #pragma unroll
     for (int nb = 0; nb < CG; ++nb) jf[kk][nb] = ws.B[(4 * kk + (lane & 3)) * BS + 8 * nb + (lane >> 2)];
+  PHASE_MARK(3);
   // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J.
-  apply_rotation<W2>(Wm, ld, mrows, I, J, lane, jf);
-  apply_rotation<W2>(Vm, ldv, vrows, I, J, lane, jf);
+  __syncwarp();  // the ring aliases B: every lane holds its J' fragments before slabs land
+  apply_rotation_async<W2>(ws, Wm, ld, mrows, I, J, lane, jf);
+  PHASE_MARK(4);
+  apply_rotation_async<W2>(ws, Vm, ldv, vrows, I, J, lane, jf);
+  PHASE_MARK(5);
   return true;
 }
 
@@ -385,13 +523,15 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     unsigned char* p = smem_raw + warp * WarpSmem<W2>::bytes();
     ws.B = reinterpret_cast<double*>(p);
     ws.S = ws.B + W2 * C::BS;
-    ws.cs = reinterpret_cast<double2*>(ws.S + W2 * C::BS);
+    ws.ring = ws.B;
+    ws.cs = reinterpret_cast<double2*>(p + WarpSmem<W2>::region());
     ws.tt = reinterpret_cast<double*>(ws.cs + W2 / 2);
     ws.pq = reinterpret_cast<int2*>(ws.tt + W2 / 2);
   }
   __shared__ int s_flags[4];
   __shared__ int s_inner[NW];
   __shared__ int s_grp[2 * NW];
+  __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
   if (tid < 4) s_flags[tid] = 0;
   if (tid < NW) s_inner[tid] = 0;
   if (tid < 2 * NW) s_grp[tid] = 0;
@@ -433,16 +573,35 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   bool converged = false;
   int my_inner = 0;
   if (!nonfinite && d.w2 == 0) {
-    // Flat Level 1: round-robin over the n_pad / w column blocks (Alg 1).
+    // Flat Level 1: round-robin over the n_pad / w column blocks (Alg 1). Pairs are
+    // scheduled by dataflow instead of a CTA barrier per step: blk_ver[b] counts the pairs block b
+    // has completed, and the pair (I, J) of global step g starts once both blocks reached g. Each
+    // warp takes its pairs in (step, pair) order, so waits only point backwards (no deadlock), and
+    // warps drift into different phases (EVD overlaps other warps' DMMA work). The arithmetic of
+    // every pair is unchanged, so the result is bitwise that of the barrier schedule.
     const int nb = np / C::W;
+    volatile int* blk_ver = s_blkver;
+    for (int b = tid; b < nb; b += T) blk_ver[b] = 0;
+    __syncthreads();
+    int gstep = 0;
     while (sweep < d.max_sweeps) {
       bool rot_any = false;
-      for (int step = 0; step < nb - 1; ++step) {
+      for (int step = 0; step < nb - 1; ++step, ++gstep) {
         for (int p = warp; p < nb / 2; p += NW) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
+          if (lane == 0) {
+            while (blk_ver[I] < gstep || blk_ver[J] < gstep) __nanosleep(20);
+          }
+          __syncwarp();
+          __threadfence_block();  // acquire: the previous owners' W / V writes are visible
           rot_any |= process_pair<W2>(ws, qm, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
+          __threadfence_block();  // release this pair's W / V writes before publishing
+          __syncwarp();
+          if (lane == 0) {
+            blk_ver[I] = gstep + 1;
+            blk_ver[J] = gstep + 1;
+          }
         }
-        __syncthreads();
       }
       ++sweep;
       if (rot_any && lane == 0) s_flags[sweep & 1] = 1;
@@ -606,3 +765,15 @@ cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int c
 }
 
 }  // namespace wcsvd
+
+#ifdef WCSVD_PHASE_PROFILE
+// Debug builds only: copy (and optionally reset) the per-phase cycle totals of the Level-1 kernel.
+extern "C" WCSVD_API int wcsvd_debug_phase_cycles(unsigned long long* out, int reset) {
+  if (cudaMemcpyFromSymbol(out, wcsvd::g_phase_cycles, sizeof(unsigned long long) * 8) != cudaSuccess) return -1;
+  if (reset) {
+    unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    cudaMemcpyToSymbol(wcsvd::g_phase_cycles, z, sizeof(z));
+  }
+  return 0;
+}
+#endif

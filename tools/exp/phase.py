@@ -1,0 +1,19 @@
+"""Run a config with the phase-profiling build and print the Level-1 cycle split."""
+import ctypes, sys
+import numpy as np, torch
+sys.path.insert(0, '.')
+import workloads
+import paper_conf_sc_xiaopxsmmlzt22_b200 as wc
+name, batch = sys.argv[1], int(sys.argv[2])
+cfg = workloads.get_config(name, batch)
+A = torch.from_numpy(np.stack(cfg.matrices())).cuda()
+L = wc.lib()
+buf = (ctypes.c_ulonglong * 8)()
+wc.svd_batched(A); torch.cuda.synchronize()
+L.wcsvd_debug_phase_cycles(buf, 1)
+wc.svd_batched(A); torch.cuda.synchronize()
+L.wcsvd_debug_phase_cycles(buf, 0)
+names = ["gram", "offtest", "evd", "ns+jfrag", "apply_A", "apply_V"]
+tot = sum(buf[i] for i in range(6))
+for i, n in enumerate(names):
+    print(f"{n:9s} {buf[i]/tot*100:5.1f}%  {buf[i]:.3e} warp-cycles")
