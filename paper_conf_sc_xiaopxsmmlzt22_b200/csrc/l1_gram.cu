@@ -342,49 +342,53 @@ struct QuadMap {
 // One inner EVD step r (round-robin over 2w indices): lanes k < w compute the
 // rotations of the step's disjoint pairs (p_k, q_k) and apply the annihilating 2x2 update to their
 // own diagonal quad; then every off-diagonal quad (k < l) of B' = G^T B G is updated from 4 loads
-// and written with its mirror (B symmetric); J <- J G in slot order.
+// and written with its mirror (B symmetric); J <- J G in slot order. rr[k] holds
+// (p BS, q BS, p, q) of pair k at this step (precomputed round-robin table). A step in which no pair
+// rotates only moves J's slots.
 template <int W2>
-__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, int r, int lane,
-                                         double tol2, const double (&x)[W2], double (&y)[W2]) {
+__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int4* __restrict__ rr,
+                                         int lane, double tol2, const double (&x)[W2], double (&y)[W2]) {
   using C = PairCfg<W2>;
-  constexpr int BS = C::BS, NPR = C::NPR;
+  constexpr int NPR = C::NPR;
   double* B = ws.B;
   bool rot = false;
   if (lane < NPR) {
-    const int p = rr_content(2 * lane, r, W2), q = rr_content(2 * lane + 1, r, W2);
-    const double bpp = B[p * BS + p], bqq = B[q * BS + q], bpq = B[p * BS + q];
+    const int4 e = rr[lane];
+    const double bpp = B[e.x + e.z], bqq = B[e.y + e.w], bpq = B[e.x + e.w];
     double c, s, t;
     rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
     ws.cs[lane] = make_double2(c, s);
-    ws.pq[lane] = make_int2(p, q);
     if (rot) {  // annihilated pair: closed-form diagonal (eq 6 analogue), exact zero off-diagonal
-      B[p * BS + p] = fma(t, bpq, bpp);
-      B[q * BS + q] = fma(-t, bpq, bqq);
-      B[p * BS + q] = 0.0;
-      B[q * BS + p] = 0.0;
+      B[e.x + e.z] = fma(t, bpq, bpp);
+      B[e.y + e.w] = fma(-t, bpq, bqq);
+      B[e.x + e.w] = 0.0;
+      B[e.y + e.z] = 0.0;
     }
   }
   const bool any = __any_sync(0xffffffffu, rot);
   __syncwarp();
-  if (any) {
+  if (!any) {
 #pragma unroll
-    for (int i = 0; i < C::QPL; ++i) {
-      if (qm.k[i] >= 0) {
-        const int2 ik = ws.pq[qm.k[i]], il = ws.pq[qm.l[i]];
-        const double2 gk = ws.cs[qm.k[i]], gl = ws.cs[qm.l[i]];
-        const double b00 = B[ik.x * BS + il.x], b01 = B[ik.x * BS + il.y];
-        const double b10 = B[ik.y * BS + il.x], b11 = B[ik.y * BS + il.y];
-        // columns (p_l, q_l): B G_l
-        const double c0 = fma(gl.y, b01, gl.x * b00), c1 = fma(-gl.y, b00, gl.x * b01);
-        const double d0 = fma(gl.y, b11, gl.x * b10), d1 = fma(-gl.y, b10, gl.x * b11);
-        // rows (p_k, q_k): G_k^T (B G_l)
-        const double e00 = fma(gk.y, d0, gk.x * c0), e01 = fma(gk.y, d1, gk.x * c1);
-        const double e10 = fma(-gk.y, c0, gk.x * d0), e11 = fma(-gk.y, c1, gk.x * d1);
-        B[ik.x * BS + il.x] = e00; B[il.x * BS + ik.x] = e00;
-        B[ik.x * BS + il.y] = e01; B[il.y * BS + ik.x] = e01;
-        B[ik.y * BS + il.x] = e10; B[il.x * BS + ik.y] = e10;
-        B[ik.y * BS + il.y] = e11; B[il.y * BS + ik.y] = e11;
-      }
+    for (int k = 0; k < W2; ++k) y[rr_dest(k, W2)] = x[k];
+    return false;
+  }
+#pragma unroll
+  for (int i = 0; i < C::QPL; ++i) {
+    if (qm.k[i] >= 0) {
+      const int4 ek = rr[qm.k[i]], el = rr[qm.l[i]];
+      const double2 gk = ws.cs[qm.k[i]], gl = ws.cs[qm.l[i]];
+      const double b00 = B[ek.x + el.z], b01 = B[ek.x + el.w];
+      const double b10 = B[ek.y + el.z], b11 = B[ek.y + el.w];
+      // columns (p_l, q_l): B G_l
+      const double c0 = fma(gl.y, b01, gl.x * b00), c1 = fma(-gl.y, b00, gl.x * b01);
+      const double d0 = fma(gl.y, b11, gl.x * b10), d1 = fma(-gl.y, b10, gl.x * b11);
+      // rows (p_k, q_k): G_k^T (B G_l)
+      const double e00 = fma(gk.y, d0, gk.x * c0), e01 = fma(gk.y, d1, gk.x * c1);
+      const double e10 = fma(-gk.y, c0, gk.x * d0), e11 = fma(-gk.y, c1, gk.x * d1);
+      B[ek.x + el.z] = e00; B[el.x + ek.z] = e00;
+      B[ek.x + el.w] = e01; B[el.y + ek.z] = e01;
+      B[ek.y + el.z] = e10; B[el.x + ek.w] = e10;
+      B[ek.y + el.w] = e11; B[el.y + ek.w] = e11;
     }
   }
   // J <- J G in slot order; outputs move to their next slots (register rename).
@@ -396,13 +400,14 @@ __device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W
     y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
   }
   __syncwarp();
-  return any;
+  return true;
 }
 
 // Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
 // rotated (A and V panels updated); counts inner sweeps into *inner.
 template <int W2>
-__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, double* Wm, int ld, int mrows,
+__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int4* __restrict__ rrtab,
+                             double* Wm, int ld, int mrows,
                              double* Vm, int ldv, int vrows, int I, int J, double tol2, int inner_cap,
                              int lane, int* inner) {
   using C = PairCfg<W2>;
@@ -438,10 +443,11 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, doub
   int isw = 0;
   for (; isw < inner_cap; ++isw) {
     // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb, slots back in order.
-    bool any = evd_step<W2>(ws, qm, 0, lane, tol2, ja, jb);
+    constexpr int NPR = W2 / 2;
+    bool any = evd_step<W2>(ws, qm, rrtab, lane, tol2, ja, jb);
     for (int r = 1; r < W2 - 1; r += 2) {
-      any |= evd_step<W2>(ws, qm, r, lane, tol2, jb, ja);
-      any |= evd_step<W2>(ws, qm, r + 1, lane, tol2, ja, jb);
+      any |= evd_step<W2>(ws, qm, rrtab + r * NPR, lane, tol2, jb, ja);
+      any |= evd_step<W2>(ws, qm, rrtab + (r + 1) * NPR, lane, tol2, ja, jb);
     }
 #pragma unroll
     for (int s = 0; s < W2; ++s) ja[s] = jb[s];
@@ -532,6 +538,12 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __shared__ int s_inner[NW];
   __shared__ int s_grp[2 * NW];
   __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
+  __shared__ int4 s_rr[(W2 - 1) * (W2 / 2)];  // EVD round-robin table: (p BS, q BS, p, q) per step, pair
+  for (int e = tid; e < (W2 - 1) * (W2 / 2); e += NW * 32) {
+    const int r = e / (W2 / 2), k = e % (W2 / 2);
+    const int p = rr_content(2 * k, r, W2), q = rr_content(2 * k + 1, r, W2);
+    s_rr[e] = make_int4(p * C::BS, q * C::BS, p, q);
+  }
   if (tid < 4) s_flags[tid] = 0;
   if (tid < NW) s_inner[tid] = 0;
   if (tid < 2 * NW) s_grp[tid] = 0;
@@ -594,7 +606,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
           }
           __syncwarp();
           __threadfence_block();  // acquire: the previous owners' W / V writes are visible
-          rot_any |= process_pair<W2>(ws, qm, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
+          rot_any |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
           __threadfence_block();  // release this pair's W / V writes before publishing
           __syncwarp();
           if (lane == 0) {
@@ -637,7 +649,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
-                  mine |= process_pair<W2>(ws, qm, Wm, mp, mp, Vm, np, np, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
+                  mine |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, np, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
                 }
                 named_bar(1 + grp, GS * 32);
               }

@@ -9,23 +9,29 @@ namespace wcsvd {
 // gamma, with tol2 = tol^2: rotate iff alpha, beta > 0 and gamma^2 > tol^2 alpha beta
 // (<=> |gamma| > tol sqrt(alpha) sqrt(beta); inputs are pre-scaled to max|a_ij| < 1 so the products
 // cannot overflow; a product that underflows to 0 means a numerically zero column: no rotation).
-// tau = (alpha - beta)/(2 gamma), t = sgn(tau)/(|tau| + sqrt(1 + tau^2)) is evaluated as
-// t = sgn(tau) 2|gamma| / (|d| + sqrt(d^2 + 4 gamma^2)), d = alpha - beta: the same number, multiplied
-// through by 2|gamma|, with one correctly-rounded reciprocal instead of three divisions.
-// sgn(0) = +1 (Z4). c = 1/sqrt(1 + t^2), s = t c. Returns true (c, s, t) if the pair rotates.
+// eq (4): tau = (alpha - beta)/(2 gamma), t = sgn(tau)/(|tau| + sqrt(1 + tau^2)), c = 1/sqrt(1+t^2),
+// s = t c, sgn(0) = +1 (Z4). Evaluated without divisions (R-ROT): with d = alpha - beta,
+// r = sqrt(d^2 + 4 gamma^2) and q = 1/sqrt(2 r (r + |d|)):
+//   c = (r + |d|) q,   s = sgn(tau) 2|gamma| q,   t = s / c = sgn(tau) 4 r |gamma| q^2,
+// the same numbers as eq (4) (multiply num/denom of t by 2|gamma|; 1/(r+|d|) = 2 r q^2), with one
+// sqrt and one rsqrt on the dependent chain. Returns true (c, s, t) if the pair rotates.
 __device__ __forceinline__ bool jacobi_rotation(double alpha, double beta, double gamma, double tol2,
                                                 double& c, double& s, double& t) {
   c = 1.0;
   s = 0.0;
   t = 0.0;
   const double ab = alpha * beta;
-  if (!(ab > 0.0) || gamma * gamma <= tol2 * ab) return false;
-  const double d = alpha - beta;
-  const double r = sqrt(fma(d, d, 4.0 * (gamma * gamma)));
-  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 1.0 : -1.0;
-  t = (sg * 2.0 * fabs(gamma)) * __drcp_rn(fabs(d) + r);
-  c = rsqrt(fma(t, t, 1.0));
-  s = t * c;
+  const double g2 = gamma * gamma;
+  if (!(ab > 0.0) || g2 <= tol2 * ab) return false;
+  const double d = alpha - beta, ad = fabs(d);
+  const double r = sqrt(fma(d, d, 4.0 * g2));
+  const double rp = r + ad;
+  const double q = rsqrt(2.0 * r * rp);
+  const double sg = (d == 0.0 || ((d > 0.0) == (gamma > 0.0))) ? 2.0 : -2.0;  // 2 sgn(tau)
+  const double sq = sg * fabs(gamma) * q;  // s
+  c = rp * q;
+  s = sq;
+  t = 2.0 * r * sq * q;  // sgn(tau) 4 r |gamma| q^2
   return true;
 }
 
