@@ -346,23 +346,40 @@ struct QuadMap {
 // (p BS, q BS, p, q) of pair k at this step (precomputed round-robin table). A step in which no pair
 // rotates only moves J's slots.
 template <int W2>
-__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int4* __restrict__ rr,
+__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int2* __restrict__ rr,
                                          int lane, double tol2, const double (&x)[W2], double (&y)[W2]) {
   using C = PairCfg<W2>;
-  constexpr int NPR = C::NPR;
+  constexpr int NPR = C::NPR, QPL = C::QPL, BS = C::BS;
   double* B = ws.B;
+  // Off-diagonal quad elements are written only by their owner lane, so they are loaded before the
+  // rotation chain of the parameter lanes and their latency overlaps it.
+  int ak[QPL], al[QPL];  // packed (p, q) of quads' row pair k and column pair l: p | q << 16
+  double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
+#pragma unroll
+  for (int i = 0; i < QPL; ++i) {
+    if (qm.k[i] >= 0) {
+      const int2 xk = rr[qm.k[i]], xl = rr[qm.l[i]];
+      ak[i] = xk.x | (xk.y << 16);
+      al[i] = xl.x | (xl.y << 16);
+      b00[i] = B[xk.x * BS + xl.x];
+      b01[i] = B[xk.x * BS + xl.y];
+      b10[i] = B[xk.y * BS + xl.x];
+      b11[i] = B[xk.y * BS + xl.y];
+    }
+  }
   bool rot = false;
   if (lane < NPR) {
-    const int4 e = rr[lane];
-    const double bpp = B[e.x + e.z], bqq = B[e.y + e.w], bpq = B[e.x + e.w];
+    const int2 pq = rr[lane];
+    const int pp = pq.x * BS + pq.x, qq = pq.y * BS + pq.y, pqo = pq.x * BS + pq.y, qpo = pq.y * BS + pq.x;
+    const double bpp = B[pp], bqq = B[qq], bpq = B[pqo];
     double c, s, t;
     rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
     ws.cs[lane] = make_double2(c, s);
     if (rot) {  // annihilated pair: closed-form diagonal (eq 6 analogue), exact zero off-diagonal
-      B[e.x + e.z] = fma(t, bpq, bpp);
-      B[e.y + e.w] = fma(-t, bpq, bqq);
-      B[e.x + e.w] = 0.0;
-      B[e.y + e.z] = 0.0;
+      B[pp] = fma(t, bpq, bpp);
+      B[qq] = fma(-t, bpq, bqq);
+      B[pqo] = 0.0;
+      B[qpo] = 0.0;
     }
   }
   const bool any = __any_sync(0xffffffffu, rot);
@@ -373,22 +390,20 @@ __device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W
     return false;
   }
 #pragma unroll
-  for (int i = 0; i < C::QPL; ++i) {
+  for (int i = 0; i < QPL; ++i) {
     if (qm.k[i] >= 0) {
-      const int4 ek = rr[qm.k[i]], el = rr[qm.l[i]];
       const double2 gk = ws.cs[qm.k[i]], gl = ws.cs[qm.l[i]];
-      const double b00 = B[ek.x + el.z], b01 = B[ek.x + el.w];
-      const double b10 = B[ek.y + el.z], b11 = B[ek.y + el.w];
       // columns (p_l, q_l): B G_l
-      const double c0 = fma(gl.y, b01, gl.x * b00), c1 = fma(-gl.y, b00, gl.x * b01);
-      const double d0 = fma(gl.y, b11, gl.x * b10), d1 = fma(-gl.y, b10, gl.x * b11);
+      const double c0 = fma(gl.y, b01[i], gl.x * b00[i]), c1 = fma(-gl.y, b00[i], gl.x * b01[i]);
+      const double d0 = fma(gl.y, b11[i], gl.x * b10[i]), d1 = fma(-gl.y, b10[i], gl.x * b11[i]);
       // rows (p_k, q_k): G_k^T (B G_l)
       const double e00 = fma(gk.y, d0, gk.x * c0), e01 = fma(gk.y, d1, gk.x * c1);
       const double e10 = fma(-gk.y, c0, gk.x * d0), e11 = fma(-gk.y, c1, gk.x * d1);
-      B[ek.x + el.z] = e00; B[el.x + ek.z] = e00;
-      B[ek.x + el.w] = e01; B[el.y + ek.z] = e01;
-      B[ek.y + el.z] = e10; B[el.x + ek.w] = e10;
-      B[ek.y + el.w] = e11; B[el.y + ek.w] = e11;
+      const int pk = ak[i] & 0xffff, qk = ak[i] >> 16, pl = al[i] & 0xffff, ql = al[i] >> 16;
+      B[pk * BS + pl] = e00; B[pl * BS + pk] = e00;
+      B[pk * BS + ql] = e01; B[ql * BS + pk] = e01;
+      B[qk * BS + pl] = e10; B[pl * BS + qk] = e10;
+      B[qk * BS + ql] = e11; B[ql * BS + qk] = e11;
     }
   }
   // J <- J G in slot order; outputs move to their next slots (register rename).
@@ -406,7 +421,7 @@ __device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W
 // Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
 // rotated (A and V panels updated); counts inner sweeps into *inner.
 template <int W2>
-__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int4* __restrict__ rrtab,
+__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int2* __restrict__ rrtab,
                              double* Wm, int ld, int mrows,
                              double* Vm, int ldv, int vrows, int I, int J, double tol2, int inner_cap,
                              int lane, int* inner) {
@@ -538,11 +553,10 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __shared__ int s_inner[NW];
   __shared__ int s_grp[2 * NW];
   __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
-  __shared__ int4 s_rr[(W2 - 1) * (W2 / 2)];  // EVD round-robin table: (p BS, q BS, p, q) per step, pair
+  __shared__ int2 s_rr[(W2 - 1) * (W2 / 2)];  // EVD round-robin table: (p, q) per step, pair
   for (int e = tid; e < (W2 - 1) * (W2 / 2); e += NW * 32) {
     const int r = e / (W2 / 2), k = e % (W2 / 2);
-    const int p = rr_content(2 * k, r, W2), q = rr_content(2 * k + 1, r, W2);
-    s_rr[e] = make_int4(p * C::BS, q * C::BS, p, q);
+    s_rr[e] = make_int2(rr_content(2 * k, r, W2), rr_content(2 * k + 1, r, W2));
   }
   if (tid < 4) s_flags[tid] = 0;
   if (tid < NW) s_inner[tid] = 0;

@@ -17,3 +17,4 @@ names = ["gram", "offtest", "evd", "ns+jfrag", "apply_A", "apply_V"]
 tot = sum(buf[i] for i in range(6))
 for i, n in enumerate(names):
     print(f"{n:9s} {buf[i]/tot*100:5.1f}%  {buf[i]:.3e} warp-cycles")
+print(f"pairs {buf[7]}, with EVD {buf[6]}; cycles/pair {tot/max(buf[7],1):.0f}; EVD cycles/call {buf[2]/max(buf[6],1):.0f}; gram/pair {buf[0]/max(buf[7],1):.0f}; apply_A/call {buf[4]/max(buf[6],1):.0f} apply_V/call {buf[5]/max(buf[6],1):.0f}")
