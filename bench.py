@@ -305,14 +305,16 @@ def main():
     achieved_tf = flops_alg / (ms_step * 1e-3) / 1e12
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
     traffic = None
-    if os.path.exists(prof):
+    if os.path.exists(prof):  # ncu --set full dram bytes of the same kernel (profiles/), per matrix x batch
         try:
-            traffic = json.load(open(prof)).get(args.config, {}).get("dram_bytes_per_launch")
+            per = json.load(open(prof)).get(args.config, {}).get("dram_bytes_per_matrix")
+            traffic = None if per is None else per * B
         except Exception:
             traffic = None
     roofline = {"bound": "alu" if dominant.startswith("l0") else "tensor", "achieved": achieved_tf,
                 "peak": FP64_PEAK_NOMINAL_TFLOPS, "unit": "TFLOP/s", "frac": achieved_tf / FP64_PEAK_NOMINAL_TFLOPS,
                 "traffic": traffic, "kernel": dominant,
+                "algorithmic_bytes": in_bytes + out_bytes,
                 "peak_note": "FP64: 148 SM x 64 FMA/clk x 2 x 1.965 GHz (MEASURED_PEAKS.json has no fp64 entry; "
                              "measured DFMA 36.5 / DMMA 37.1 TF/s, profiles/peaks_fp64_r01.json)",
                 "flops": "textbook F_tb(M,N)=N(N-1)/2(8M+6N) x sweeps used, summed over the batch"}
