@@ -606,7 +606,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     // warps drift into different phases (EVD overlaps other warps' DMMA work). The arithmetic of
     // every pair is unchanged, so the result is bitwise that of the barrier schedule.
     const int nb = np / C::W;
-    volatile int* blk_ver = s_blkver;
+    int* blk_ver = s_blkver;
     for (int b = tid; b < nb; b += T) blk_ver[b] = 0;
     __syncthreads();
     int gstep = 0;
@@ -615,17 +615,17 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
       for (int step = 0; step < nb - 1; ++step, ++gstep) {
         for (int p = warp; p < nb / 2; p += NW) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
-          if (lane == 0) {
-            while (blk_ver[I] < gstep || blk_ver[J] < gstep) __nanosleep(20);
+          if (lane == 0) {  // acquire: relaxed atomic reads, then a fence
+            while (atomicAdd(&blk_ver[I], 0) < gstep || atomicAdd(&blk_ver[J], 0) < gstep) __nanosleep(20);
           }
           __syncwarp();
-          __threadfence_block();  // acquire: the previous owners' W / V writes are visible
+          __threadfence_block();  // the previous owners' W / V writes are visible to every lane
           rot_any |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
-          __threadfence_block();  // release this pair's W / V writes before publishing
-          __syncwarp();
+          __syncwarp();           // every lane's W / V writes precede ...
+          __threadfence_block();  // ... this fence, then the release (relaxed atomic store)
           if (lane == 0) {
-            blk_ver[I] = gstep + 1;
-            blk_ver[J] = gstep + 1;
+            atomicExch(&blk_ver[I], gstep + 1);
+            atomicExch(&blk_ver[J], gstep + 1);
           }
         }
       }

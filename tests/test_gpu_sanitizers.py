@@ -1,0 +1,26 @@
+"""T8: compute-sanitizer memcheck / racecheck / synccheck / initcheck on a small mixed
+batch covering the Level-0 variants, the Level-1 Gram path (w = 8 and 16, dataflow pair scheduling,
+cp.async slab rings) and the W-cycle path."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+
+
+@pytest.mark.parametrize("tool,mode", [("memcheck", "mixed"), ("racecheck", "mixed"), ("racecheck", "wcycle"),
+                                       ("synccheck", "mixed"), ("initcheck", "mixed")])
+def test_sanitizer_clean(tool, mode):
+    if not os.path.exists(SAN):
+        pytest.skip("compute-sanitizer not available")
+    out = subprocess.run([SAN, "--tool", tool, "--error-exitcode", "3", sys.executable,
+                          os.path.join(ROOT, "tools", "sanitize_case.py"), mode],
+                         cwd=ROOT, capture_output=True, text=True, timeout=900)
+    text = out.stdout + out.stderr
+    assert out.returncode == 0, text[-3000:]
+    assert "info" in text
