@@ -142,6 +142,7 @@ def cpu_baseline(cfg_name, sizes_idx, make, seconds_target=15.0, sample=None):
     t0 = time.perf_counter()
     _, _, _, info = oracle.svd_batch(mats, precision="d", threads=cores, lib_path=lib)
     dt = time.perf_counter() - t0
+    cores = oracle.threads_in_effect(lib)
     return {"value": len(sel) / dt, "unit": "matrices/s", "cores": cores, "kind": "oracle",
             "sample": f"{len(sel)} of the config's matrices (every {step}th), cyclic one-sided Jacobi, "
                       f"oracle/oracle.c T=double, OpenMP x{cores}; {dt:.1f} s; mean sweeps {float(np.mean(info)):.2f}"}
@@ -168,6 +169,7 @@ def run_reference(args, world, rank):
         if s >= args.warmup:
             times.append(time.perf_counter() - t0)
     value = n * len(times) / sum(times)
+    cores = oracle.threads_in_effect(lib)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "matrices/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
@@ -190,11 +192,16 @@ def main():
 
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (the library has no CPU fallback)")
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % ndev  # == local on a real box (one process per GPU)
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if ndev >= world:
+            dist.init_process_group("nccl", device_id=dev)
+        else:  # ranks sharing a GPU (1-GPU development box): NCCL refuses duplicate devices
+            dist.init_process_group("gloo")
 
     base, idx, sizes, make = local_config(args.config, args.batch, rank)
     B = len(idx)
@@ -240,7 +247,7 @@ def main():
     barrier()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    with ClockSampler(local_dev) as clk:
         ev0.record(stream)
         for _ in range(args.steps):
             res = call(A)
@@ -249,7 +256,7 @@ def main():
     ms = ev0.elapsed_time(ev1)
     if world > 1:
         import torch.distributed as dist
-        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        t = torch.tensor([ms], dtype=torch.float64, device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     ms_step = ms / args.steps
@@ -287,7 +294,7 @@ def main():
     e_ms = ee0.elapsed_time(ee1)
     if world > 1:
         import torch.distributed as dist
-        t = torch.tensor([e_ms], device=dev, dtype=torch.float64)
+        t = torch.tensor([e_ms], dtype=torch.float64, device=dev if dist.get_backend() == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e_ms = float(t.item())
     e2e_value = world * B * e_steps / (e_ms * 1e-3)

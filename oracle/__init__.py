@@ -66,12 +66,19 @@ def _lib(path: str | None = None) -> ctypes.CDLL:
     lib.oracle_syevj_ld.argtypes = [I, P, D, I, P, P]
     lib.oracle_syevj_ld.restype = I
     lib.oracle_ldbl_mant_dig.restype = I
+    lib.oracle_set_threads.argtypes = [I]
+    lib.oracle_set_threads.restype = None
+    lib.oracle_get_threads.restype = I
     _lib_cache[path] = lib
     return lib
 
 
 def ldbl_mant_dig() -> int:
     return _lib().oracle_ldbl_mant_dig()
+
+
+def threads_in_effect(lib_path: str | None = None) -> int:
+    return _lib(lib_path).oracle_get_threads()
 
 
 @dataclass
@@ -124,7 +131,7 @@ def svd_batch(As: list[np.ndarray], tol: float = 0.0, max_sweeps: int = 0, preci
     order = np.argsort(-cost, kind="stable").astype(np.int32)
     arr = lambda lst: (ctypes.c_void_p * B)(*[_ptr(x) for x in lst])
     if threads is not None:
-        os.environ["OMP_NUM_THREADS"] = str(threads)
+        lib.oracle_set_threads(int(threads))
     fn = getattr(lib, f"oracle_svd_batch_{precision}")
     fn(B, _ptr(ms), _ptr(ns), arr(Afs), _ptr(ms), float(tol), int(max_sweeps), arr(Ss), arr(Us), arr(Vs),
        _ptr(info), _ptr(order))

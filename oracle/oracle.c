@@ -18,6 +18,7 @@
  * and LAPACK svd cross-check (P6), rank-deficient completion (Z14). Build: gcc -O2 -fopenmp -shared.
  */
 #include <math.h>
+#include <omp.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -108,6 +109,11 @@ int oracle_syevj_ld(int n, const double* B_in, double tol_in, int max_sweeps, do
   free(B); free(J);
   return converged ? sweeps : -1;
 }
+
+/* OpenMP thread count of the batched drivers (set explicitly: launchers such as torchrun export
+ * OMP_NUM_THREADS=1), and the count actually in effect. */
+void oracle_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
+int oracle_get_threads(void) { return omp_get_max_threads(); }
 
 /* Mantissa bits of long double on this host (tests assert 64 for the x87 format). */
 int oracle_ldbl_mant_dig(void) { return __LDBL_MANT_DIG__; }
