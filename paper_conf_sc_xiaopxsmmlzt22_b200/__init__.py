@@ -141,7 +141,8 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
 
 
 def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = True,
-                return_info: bool = False, out=None, **kw):
+                return_info: bool = False, out=None, compute_u: bool | None = None,
+                compute_v: bool | None = None, **kw):
     """Batched economy SVD of fp64 CUDA tensors on the current stream.
 
     A: tensor [B, m, n] (contiguous) or a sequence of 2-D tensors (sizes may differ).
@@ -149,8 +150,14 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
     V [B, n, k] (U, V are transposed views); for a list, lists of tensors. With return_info,
     also the per-matrix int32 info tensor (sweeps, -1 not converged, -2 non-finite).
     ``out`` = (S, Ubuf, Vbuf) preallocated as returned by a previous call (batched form only).
+    ``compute_u`` / ``compute_v`` (default: ``compute_uv``) select the factors; an unrequested factor
+    is returned as None and, when it is the square one, is not accumulated at all (values / U-only
+    mode; vector signs then follow the returned factor).
     """
     import torch
+
+    cu = compute_uv if compute_u is None else compute_u
+    cv = compute_uv if compute_v is None else compute_v
 
     if not torch.cuda.is_available():
         raise WcsvdError(WCSVD_ECUDA, "no CUDA device (this library has no CPU fallback)")
@@ -166,21 +173,21 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
             S, Ubuf, Vbuf = out
         else:
             S = torch.empty(B, k, dtype=torch.float64, device=dev)
-            Ubuf = torch.empty(B, k, m, dtype=torch.float64, device=dev) if compute_uv else None
-            Vbuf = torch.empty(B, k, n, dtype=torch.float64, device=dev) if compute_uv else None
+            Ubuf = torch.empty(B, k, m, dtype=torch.float64, device=dev) if cu else None
+            Vbuf = torch.empty(B, k, n, dtype=torch.float64, device=dev) if cv else None
         info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
         idx = np.arange(B, dtype=np.uint64)
         a_ptr = A.data_ptr() + idx * np.uint64(8 * m * n)
         s_ptr = S.data_ptr() + idx * np.uint64(8 * k)
         # column-major view: the library factors A^T (n x m, lda = n); its "U" (n x k) is our V,
         # its "V" (m x k) is our U.
-        u_ptr = (Vbuf.data_ptr() + idx * np.uint64(8 * k * n)) if compute_uv else None
-        v_ptr = (Ubuf.data_ptr() + idx * np.uint64(8 * k * m)) if compute_uv else None
+        u_ptr = (Vbuf.data_ptr() + idx * np.uint64(8 * k * n)) if Vbuf is not None else None
+        v_ptr = (Ubuf.data_ptr() + idx * np.uint64(8 * k * m)) if Ubuf is not None else None
         svd_batched_raw(np.full(B, n), np.full(B, m), a_ptr, np.full(B, n), s_ptr, u_ptr, v_ptr,
                         tol=tol, max_sweeps=max_sweeps, stream=stream,
                         info_ptr=info.data_ptr() if info is not None else 0, **kw)
-        U = Ubuf.transpose(1, 2) if compute_uv else None
-        V = Vbuf.transpose(1, 2) if compute_uv else None
+        U = Ubuf.transpose(1, 2) if Ubuf is not None else None
+        V = Vbuf.transpose(1, 2) if Vbuf is not None else None
         return (S, U, V, info) if return_info else (S, U, V)
     # list of 2-D tensors
     As = [a.contiguous() for a in A]
@@ -195,14 +202,14 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
     ns = [a.shape[1] for a in As]
     ks = [min(x, y) for x, y in zip(ms, ns)]
     Ss = [torch.empty(k, dtype=torch.float64, device=dev) for k in ks]
-    Ub = [torch.empty(k, mm, dtype=torch.float64, device=dev) for k, mm in zip(ks, ms)] if compute_uv else None
-    Vb = [torch.empty(k, nn, dtype=torch.float64, device=dev) for k, nn in zip(ks, ns)] if compute_uv else None
+    Ub = [torch.empty(k, mm, dtype=torch.float64, device=dev) for k, mm in zip(ks, ms)] if cu else None
+    Vb = [torch.empty(k, nn, dtype=torch.float64, device=dev) for k, nn in zip(ks, ns)] if cv else None
     info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
     svd_batched_raw(ns, ms, [a.data_ptr() for a in As], ns, [s.data_ptr() for s in Ss],
-                    [v.data_ptr() for v in Vb] if compute_uv else None,
-                    [u.data_ptr() for u in Ub] if compute_uv else None,
+                    [v.data_ptr() for v in Vb] if Vb is not None else None,
+                    [u.data_ptr() for u in Ub] if Ub is not None else None,
                     tol=tol, max_sweeps=max_sweeps, stream=stream,
                     info_ptr=info.data_ptr() if info is not None else 0, **kw)
-    Us = [u.T for u in Ub] if compute_uv else None
-    Vs = [v.T for v in Vb] if compute_uv else None
+    Us = [u.T for u in Ub] if Ub is not None else None
+    Vs = [v.T for v in Vb] if Vb is not None else None
     return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)

@@ -84,7 +84,7 @@ size_t l1_bytes(const wcsvd_plan_t& p) {
 }
 
 struct Bucket {
-  int path, variant;
+  int path, variant, withv;
   std::vector<int> members;  // batch indices, largest cost first
   int maxM = 0;
 };
@@ -194,13 +194,18 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     const int rc = plan_one(m[b], n[b], force_path, force_w, &plans[b]);
     if (rc != WCSVD_OK) return rc;
   }
+  // V_x (the square factor) is accumulated only if it is requested: as V when m >= n, as U when
+  // m < n (§8(f4) values / U-only mode otherwise; the iteration itself is unchanged).
+  std::vector<int> withv(batch);
+  for (int b = 0; b < batch; ++b)
+    withv[b] = plans[b].swapped ? (U && U[b] ? 1 : 0) : (V && V[b] ? 1 : 0);
   std::vector<Bucket> buckets;
   for (int b = 0; b < batch; ++b) {
     Bucket* bk = nullptr;
     for (auto& x : buckets)
-      if (x.path == plans[b].path && x.variant == plans[b].variant) bk = &x;
+      if (x.path == plans[b].path && x.variant == plans[b].variant && x.withv == withv[b]) bk = &x;
     if (!bk) {
-      buckets.push_back(Bucket{plans[b].path, plans[b].variant, {}, 0});
+      buckets.push_back(Bucket{plans[b].path, plans[b].variant, withv[b], {}, 0});
       bk = &buckets.back();
     }
     bk->members.push_back(b);
@@ -272,6 +277,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     d.inner_cap2 = (opts && opts->wcycle_sweeps > 0) ? opts->wcycle_sweeps : 2;
     d.idx = b;
     d.status = d_status;
+    d.withv = withv[b];
     if (p.path != WCSVD_PATH_L0) {
       d.W = reinterpret_cast<double*>(ws + l1_off[b]);
       d.Vw = d.W + (size_t)p.m_pad * p.n_pad;
@@ -311,7 +317,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     const int cnt = (int)bk.members.size();
     cudaStream_t st = (nbk > 1) ? side[i] : stream;
     if (bk.path == WCSVD_PATH_L0)
-      e = launch_l0(bk.variant, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
+      e = launch_l0(bk.variant, bk.withv, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
       e = launch_l1(bk.variant, d_descs, d_order + bucket_off[i], cnt, st);
     if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);

@@ -65,6 +65,7 @@ struct MatDesc {
   int m_pad, n_pad, w, w2;
   int max_sweeps, inner_cap;
   int inner_cap2;  // W-cycle: cap on Level-2 sweeps per super-pair
+  int withv;       // 1: accumulate V_x (requested as V, or as U when swapped); 0: values / U-only mode
   int idx;      // index of this matrix in the caller's batch (info / status arrays)
   int* status;  // internal per-matrix status flags (workspace), e.g. kNeedsCompletion
 };

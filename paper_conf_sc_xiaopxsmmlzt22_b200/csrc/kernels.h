@@ -25,7 +25,7 @@ enum L1Variant {
 
 cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
 
-cudaError_t launch_l0(int variant, const MatDesc* descs, const int* order, int count, int maxM,
+cudaError_t launch_l0(int variant, int withv, const MatDesc* descs, const int* order, int count, int maxM,
                       cudaStream_t stream);
 
 }  // namespace wcsvd

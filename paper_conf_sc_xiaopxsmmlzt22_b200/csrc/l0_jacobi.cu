@@ -166,11 +166,11 @@ __device__ __forceinline__ void l0_sweep(L0Ctx& cx, double (&x)[R][NP / G], doub
 }  // namespace
 
 // Shared-memory bytes of one CTA (must match the carve-up in the kernel).
-template <int NP, int G, int R>
+template <int NP, int G, int R, bool WITHV>
 size_t l0_smem_bytes(int M, int threads) {
   const int RW4 = ((M + R - 1) / R + 3) / 4 * 4;
   const int PS = NP / 2 + 1;
-  const int RV = NP / R;
+  const int RV = WITHV ? NP / R : RW4;  // rows of the sign-rule scratch (V rows, or X rows)
   const int LP = NP / G / 2;
   const int NW = threads / 32;
   return sizeof(double) * 6 * (size_t)RW4 * PS                         // partials, 2 parities
@@ -181,13 +181,13 @@ size_t l0_smem_bytes(int M, int threads) {
 // One CTA per matrix. Thread t: group g = t % G, row-thread rt = t / G. Row-threads [0, RW) hold
 // rows rt*R .. rt*R+R-1 of X; row-threads [RW, RW+RV) hold rows of V (RV = NP/R); the rest (to a
 // multiple of 32) hold zeros and only take part in shuffles.
-template <int NP, int G, int R, int MAXT>
+template <int NP, int G, int R, int MAXT, bool WITHV>
 __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restrict__ descs,
                                                         const int* __restrict__ order) {
   constexpr int NL = NP / G;
   constexpr int LP = NL / 2;
   constexpr int NPAIR = NP / 2;
-  constexpr int RV = NP / R;
+  constexpr int RV = WITHV ? NP / R : 0;  // V row-threads (none in the values / U-only mode, §8(f4))
   const MatDesc d = descs[order[blockIdx.x]];
   const int M = d.M, N = d.N;
   const int RW = (M + R - 1) / R;
@@ -207,8 +207,9 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   double* s_nrmw = reinterpret_cast<double*>(s_csw + NWARP * G * (LP + 1));  // [NWARP][2][NP]
   double* s_sig = s_nrmw + NWARP * 2 * NP;                                // [NP]
   double* s_sgn = s_sig + NP;                                             // [NP]
-  double* s_vbest = s_sgn + NP;                                           // [RV][NP]
-  int* s_rank = reinterpret_cast<int*>(s_vbest + RV * NP);                // [NP]
+  const int SR = WITHV ? RV : RW4;                                        // sign-rule rows
+  double* s_vbest = s_sgn + NP;                                           // [SR][NP]
+  int* s_rank = reinterpret_cast<int*>(s_vbest + SR * NP);                // [NP]
   int* s_flags = s_rank + NP;                                             // [8]
   unsigned long long* s_max = reinterpret_cast<unsigned long long*>(s_flags + 4);
   if (tid < 4) s_flags[tid] = 0;
@@ -309,14 +310,16 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
       s_part[(col < NPAIR ? 0 : RW4) * PS + rt * PS + (col % NPAIR)] = a;
     }
   }
-  if (isV) {
+  // Z15 sign rule: the largest-|.| entry (first on ties) of each column of the square factor V_x is
+  // made positive; without V (values / U-only mode) the rule is applied to the columns of X instead.
+  if (WITHV ? isV : isW) {
 #pragma unroll
     for (int l = 0; l < NL; ++l) {
       double best = 0.0;
 #pragma unroll
       for (int r = 0; r < R; ++r)
         if (fabs(xa[r][l]) > fabs(best)) best = xa[r][l];
-      s_vbest[(rt - RW) * NP + g * NL + l] = best;
+      s_vbest[(rt - (WITHV ? RW : 0)) * NP + g * NL + l] = best;
     }
   }
   __syncthreads();
@@ -329,7 +332,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
     }
     s_sig[j] = sqrt((a4[0] + a4[1]) + (a4[2] + a4[3]));  // of the pre-scaled X
     double best = 0.0;
-    for (int i = 0; i < RV; ++i) {
+    for (int i = 0; i < (WITHV ? RV : RW); ++i) {
       const double v = s_vbest[i * NP + j];
       if (fabs(v) > fabs(best)) best = v;
     }
@@ -406,40 +409,41 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
 }
 
 // ---- launcher ----
-template <int NP, int G, int R, int MAXT>
+template <int NP, int G, int R, int MAXT, bool WITHV>
 static cudaError_t launch_l0_t(const MatDesc* descs, const int* order, int count, int maxM,
                                cudaStream_t stream) {
   const int RW = (maxM + R - 1) / R;
-  int threads = (RW + NP / R) * G;
+  int threads = (RW + (WITHV ? NP / R : 0)) * G;
   threads = (threads + 31) / 32 * 32;
   if (threads > MAXT) return cudaErrorInvalidConfiguration;
-  const size_t smem = l0_smem_bytes<NP, G, R>(maxM, threads);
-  auto kern = l0_jacobi_kernel<NP, G, R, MAXT>;
+  const size_t smem = l0_smem_bytes<NP, G, R, WITHV>(maxM, threads);
+  auto kern = l0_jacobi_kernel<NP, G, R, MAXT, WITHV>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<count, threads, smem, stream>>>(descs, order);
   return cudaGetLastError();
 }
 
-int l0_max_threads(int variant) {
+template <bool WITHV>
+static cudaError_t launch_l0_v(int variant, const MatDesc* descs, const int* order, int count, int maxM,
+                               cudaStream_t stream) {
   switch (variant) {
-    case kL0_32s: return 512;
-    default: return 256;
+    case kL0_8:   return launch_l0_t<8, 1, 8, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_16:  return launch_l0_t<16, 2, 8, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_32:  return launch_l0_t<32, 2, 4, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_32s: return launch_l0_t<32, 2, 1, 512, WITHV>(descs, order, count, maxM, stream);
+    case kL0_48:  return launch_l0_t<48, 2, 2, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_64:  return launch_l0_t<64, 4, 4, 256, WITHV>(descs, order, count, maxM, stream);
+    default: return cudaErrorInvalidValue;
   }
 }
 
-// Variant table (planner ids). E = R * NP / G doubles per thread.
-cudaError_t launch_l0(int variant, const MatDesc* descs, const int* order, int count, int maxM,
+// Variant table (planner ids). E = R * NP / G doubles per thread. withv = 0: V_x is not accumulated
+// (it is not requested; §8(f4) values / U-only mode) -- half the threads and registers per matrix.
+cudaError_t launch_l0(int variant, int withv, const MatDesc* descs, const int* order, int count, int maxM,
                       cudaStream_t stream) {
-  switch (variant) {
-    case kL0_8:   return launch_l0_t<8, 1, 8, 256>(descs, order, count, maxM, stream);
-    case kL0_16:  return launch_l0_t<16, 2, 8, 256>(descs, order, count, maxM, stream);
-    case kL0_32:  return launch_l0_t<32, 2, 4, 256>(descs, order, count, maxM, stream);
-    case kL0_32s: return launch_l0_t<32, 2, 1, 512>(descs, order, count, maxM, stream);
-    case kL0_48:  return launch_l0_t<48, 2, 2, 256>(descs, order, count, maxM, stream);
-    case kL0_64:  return launch_l0_t<64, 4, 4, 256>(descs, order, count, maxM, stream);
-    default: return cudaErrorInvalidValue;
-  }
+  return withv ? launch_l0_v<true>(variant, descs, order, count, maxM, stream)
+               : launch_l0_v<false>(variant, descs, order, count, maxM, stream);
 }
 
 }  // namespace wcsvd

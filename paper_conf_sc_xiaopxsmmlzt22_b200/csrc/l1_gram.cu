@@ -578,7 +578,9 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     }
     Wm[e] = v;
   }
-  for (size_t e = tid; e < (size_t)np * np; e += T) Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
+  if (d.withv)
+    for (size_t e = tid; e < (size_t)np * np; e += T) Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
+  const int vrows = d.withv ? np : 0;  // values / U-only mode: V_x is not accumulated (§8(f4))
   if (bad) atomicOr(&s_flags[2], 1);
   if (amax > 0.0) atomicMax(&s_max, (unsigned long long)__double_as_longlong(amax));
   __syncthreads();
@@ -620,7 +622,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
           }
           __syncwarp();
           __threadfence_block();  // the previous owners' W / V writes are visible to every lane
-          rot_any |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, np, I, J, tol2, d.inner_cap, lane, &my_inner);
+          rot_any |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
           __syncwarp();           // every lane's W / V writes precede ...
           __threadfence_block();  // ... this fence, then the release (relaxed atomic store)
           if (lane == 0) {
@@ -663,7 +665,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
-                  mine |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, np, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
+                  mine |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
                 }
                 named_bar(1 + grp, GS * 32);
               }
@@ -701,10 +703,12 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     double a = 0.0;
     for (int r = lane; r < M; r += 32) a = fma(col[r], col[r], a);
     for (int off = 16; off > 0; off >>= 1) a += __shfl_xor_sync(0xffffffffu, a, off);
-    const double* vc = Vm + (size_t)j * np;
+    // Z15 sign rule on the square factor V_x; without V (values / U-only mode) on the columns of X.
+    const double* vc = d.withv ? Vm + (size_t)j * np : col;
+    const int vlen = d.withv ? N : M;
     double best = 0.0;
     int bi = 0x7fffffff;
-    for (int i = lane; i < N; i += 32) {
+    for (int i = lane; i < vlen; i += 32) {
       const double v = vc[i];
       if (fabs(v) > fabs(best)) { best = v; bi = i; }
     }
