@@ -31,7 +31,7 @@ int l0_variant(int M, int N) {
     return ((M + 3) / 4 + 8) * 2 <= 256 ? kL0_32 : 0;
   }
   if (N <= 48) return ((M + 1) / 2 + 24) * 2 <= 256 ? kL0_48 : 0;
-  if (N <= 64) return ((M + 1) / 2 + 32) * 2 <= 256 ? kL0_64 : 0;
+  if (N <= 64) return ((M + 7) / 8 + 8) * 8 <= 256 ? kL0_64 : 0;  // G = 8, R = 8
   return 0;
 }
 

@@ -13,7 +13,7 @@ enum L0Variant {
   kL0_32 = 3,   // NP=32, G=2, R=4
   kL0_32s = 4,  // NP=32, G=2, R=1 (latency-bound small batches)
   kL0_48 = 5,   // NP=48, G=2, R=2
-  kL0_64 = 6,   // NP=64, G=2, R=2
+  kL0_64 = 6,   // NP=64, G=8, R=8
 };
 
 // Level-1 Gram-path variants (pair panel width 2w, warps per CTA).

@@ -433,7 +433,7 @@ static cudaError_t launch_l0_v(int variant, const MatDesc* descs, const int* ord
     case kL0_32:  return launch_l0_t<32, 2, 4, 256, WITHV>(descs, order, count, maxM, stream);
     case kL0_32s: return launch_l0_t<32, 2, 1, 512, WITHV>(descs, order, count, maxM, stream);
     case kL0_48:  return launch_l0_t<48, 2, 2, 256, WITHV>(descs, order, count, maxM, stream);
-    case kL0_64:  return launch_l0_t<64, 4, 4, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_64:  return launch_l0_t<64, 8, 8, 256, WITHV>(descs, order, count, maxM, stream);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -33,7 +33,7 @@ namespace {
 
 #ifdef WCSVD_PHASE_PROFILE
 // Debug builds only (-DWCSVD_PHASE_PROFILE): per-phase clock64() totals, lane 0 of every warp.
-__device__ unsigned long long g_phase_cycles[8];
+__device__ unsigned long long g_phase_cycles[12];
 #define PHASE_T0() long long _pt = clock64()
 #define PHASE_MARK(i)                                                        \
   do {                                                                       \
@@ -41,9 +41,14 @@ __device__ unsigned long long g_phase_cycles[8];
     if ((threadIdx.x & 31) == 0) atomicAdd(&g_phase_cycles[i], (unsigned long long)(_pn - _pt)); \
     _pt = _pn;                                                               \
   } while (0)
+#define PHASE_COUNT(i)                                                       \
+  do {                                                                       \
+    if ((threadIdx.x & 31) == 0) atomicAdd(&g_phase_cycles[i], 1ull);        \
+  } while (0)
 #else
 #define PHASE_T0() (void)0
 #define PHASE_MARK(i) (void)0
+#define PHASE_COUNT(i) (void)0
 #endif
 
 __device__ __forceinline__ void named_bar(int id, int count) {
@@ -385,6 +390,7 @@ __device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W
   const bool any = __any_sync(0xffffffffu, rot);
   __syncwarp();
   if (!any) {
+    PHASE_COUNT(8);  // profiling builds: rotation-free EVD steps
 #pragma unroll
     for (int k = 0; k < W2; ++k) y[rr_dest(k, W2)] = x[k];
     return false;
@@ -449,6 +455,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, cons
     }
   }
   PHASE_MARK(1);
+  PHASE_COUNT(7);
   if (!__any_sync(0xffffffffu, need)) return false;
   // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, J accumulated in slot order.
   double ja[W2], jb[W2];
@@ -471,6 +478,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, cons
   }
   *inner += isw + (isw < inner_cap ? 1 : 0);
   PHASE_MARK(2);
+  PHASE_COUNT(6);
   if (!rotated) return false;
   // Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2.
   if (lane < W2) {
@@ -799,9 +807,9 @@ cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int c
 #ifdef WCSVD_PHASE_PROFILE
 // Debug builds only: copy (and optionally reset) the per-phase cycle totals of the Level-1 kernel.
 extern "C" WCSVD_API int wcsvd_debug_phase_cycles(unsigned long long* out, int reset) {
-  if (cudaMemcpyFromSymbol(out, wcsvd::g_phase_cycles, sizeof(unsigned long long) * 8) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(out, wcsvd::g_phase_cycles, sizeof(unsigned long long) * 12) != cudaSuccess) return -1;
   if (reset) {
-    unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long z[12] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     cudaMemcpyToSymbol(wcsvd::g_phase_cycles, z, sizeof(z));
   }
   return 0;

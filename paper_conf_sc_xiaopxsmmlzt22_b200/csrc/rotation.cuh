@@ -35,4 +35,31 @@ __device__ __forceinline__ bool jacobi_rotation(double alpha, double beta, doubl
   return true;
 }
 
+// Same rotation with the angle evaluated in fp32 (R-ROT32). The threshold test and d
+// are fp64; (d, gamma) are rescaled by an exact power of two into fp32 range (t is homogeneous of
+// degree 0 in them), t is formed in fp32 (~1e-7 relative), then c = 1/sqrt(1 + t^2) and s = t c are
+// fp64, so the rotation applied is orthogonal to fp64 rounding; only its angle differs from the
+// exact eq (4) angle by ~1e-7 relative, which changes the pace of convergence, not the result.
+// Updates that follow must use the general forms valid for any (c, s) (eq 6 as printed; the full
+// 2x2 two-sided update), not the closed forms that assume the exact angle.
+__device__ __forceinline__ bool jacobi_rotation_f32(double alpha, double beta, double gamma, double tol2,
+                                                    double& c, double& s) {
+  c = 1.0;
+  s = 0.0;
+  const double ab = alpha * beta;
+  const double g2 = gamma * gamma;
+  if (!(ab > 0.0) || g2 <= tol2 * ab) return false;
+  const double d = alpha - beta;
+  const double mx = fmax(fabs(d), fabs(gamma));
+  const int ex = (int)((unsigned long long)__double_as_longlong(mx) >> 52) & 0x7ff;  // mx > 0, normal
+  const double sc = __longlong_as_double((long long)(2046 - ex) << 52);              // 2^-(ex-1023)
+  const float df = __double2float_rn(d * sc), gf = __double2float_rn(gamma * sc);
+  const float r = sqrtf(fmaf(df, df, 4.0f * gf * gf));
+  const float sg = (df == 0.0f || ((df > 0.0f) == (gf > 0.0f))) ? 2.0f : -2.0f;
+  const double t = (double)(sg * fabsf(gf) * __frcp_rn(fabsf(df) + r));
+  c = rsqrt(fma(t, t, 1.0));
+  s = t * c;
+  return true;
+}
+
 }  // namespace wcsvd

@@ -8,7 +8,7 @@ name, batch = sys.argv[1], int(sys.argv[2])
 cfg = workloads.get_config(name, batch)
 A = torch.from_numpy(np.stack(cfg.matrices())).cuda()
 L = wc.lib()
-buf = (ctypes.c_ulonglong * 8)()
+buf = (ctypes.c_ulonglong * 12)()
 wc.svd_batched(A); torch.cuda.synchronize()
 L.wcsvd_debug_phase_cycles(buf, 1)
 wc.svd_batched(A); torch.cuda.synchronize()
@@ -17,4 +17,5 @@ names = ["gram", "offtest", "evd", "ns+jfrag", "apply_A", "apply_V"]
 tot = sum(buf[i] for i in range(6))
 for i, n in enumerate(names):
     print(f"{n:9s} {buf[i]/tot*100:5.1f}%  {buf[i]:.3e} warp-cycles")
+print(f"EVD steps {buf[6]*31}, rotation-free {buf[8]} ({100*buf[8]/max(buf[6]*31,1):.1f}%)")
 print(f"pairs {buf[7]}, with EVD {buf[6]}; cycles/pair {tot/max(buf[7],1):.0f}; EVD cycles/call {buf[2]/max(buf[6],1):.0f}; gram/pair {buf[0]/max(buf[7],1):.0f}; apply_A/call {buf[4]/max(buf[6],1):.0f} apply_V/call {buf[5]/max(buf[6],1):.0f}")
