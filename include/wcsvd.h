@@ -104,6 +104,19 @@ WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const doub
                      double* const* S, double* const* U, double* const* V, double tol,
                      int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
 
+/* wcsvd_batched_f32 / _f32_ex -- the fp32 variant: same arguments, layout,
+ * ownership, errors and determinism as wcsvd_batched, with float data. tol <= 0 -> sqrt(max(m,n)) *
+ * 2^-24. Level-0 matrices are iterated in fp32 throughout; Level-1 (Gram path) matrices are iterated
+ * by the fp64 DMMA kernel on an fp64 working copy (sm_100a has no full-precision fp32 MMA) and
+ * rounded to fp32 at finalisation. Accuracy targets (north_star): sigma 1e-5, residual 1e-5,
+ * orthogonality 1e-4, all relative. */
+WCSVD_API int wcsvd_batched_f32(int batch, const int* m, const int* n, const float* const* A, const int* lda,
+                                float* const* S, float* const* U, float* const* V, float tol, int max_sweeps,
+                                wcsvd_stream_t stream);
+WCSVD_API int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const float* const* A,
+                                   const int* lda, float* const* S, float* const* U, float* const* V,
+                                   float tol, int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
+
 /* Bytes of device workspace wcsvd_batched_ex needs for this batch (host-only, no CUDA call). */
 WCSVD_API size_t wcsvd_workspace_size(int batch, const int* m, const int* n);
 

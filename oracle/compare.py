@@ -83,7 +83,15 @@ def orthogonality(Q) -> float:
     return float(np.abs(Q_.T @ Q_ - np.eye(k, dtype=dt)).max()) if k else 0.0
 
 
-def compare(A, S, U, V, S_ref, U_ref, V_ref, check_vectors: bool = True) -> Parity:
+# fp32 (north_star gives sigma / residual / orthogonality only; the vector floors follow from a backward
+# error of ~1e-6 ||A|| after ~300 fp32 rotations per column: angle ~1e-3 at relative gaps ~1e-3).
+FP32_BARS = dict(sigma_tol=1e-5, resid_tol=1e-5, ortho_tol=1e-4, vec_tol=1e-5, proj_tol=1e-3)
+
+
+def compare(A, S, U, V, S_ref, U_ref, V_ref, check_vectors: bool = True, u: float = 2.0 ** -53,
+            vec_tol: float = VEC_TOL, proj_tol: float = PROJ_TOL) -> Parity:
+    """u: unit roundoff of the arithmetic under test (2^-53 fp64, 2^-24 fp32) for the R-VEC bound;
+    vec_tol / proj_tol: the floors the returned errors are scaled against (Parity.ok() bars)."""
     A = np.asarray(A, dtype=np.float64)
     S = np.asarray(S, dtype=np.float64)
     S_ref = np.asarray(S_ref, dtype=np.float64)
@@ -110,13 +118,13 @@ def compare(A, S, U, V, S_ref, U_ref, V_ref, check_vectors: bool = True) -> Pari
                 delta = gap
                 if X.shape[0] > k:  # the long factor: its null space competes (Wedin)
                     delta = min(delta, S_ref[b - 1])
-                theta = 64 * 2.0 ** -53 * s1 / delta if delta > 0 else np.inf
+                theta = 64 * u * s1 / delta if delta > 0 else np.inf
                 if b - a == 1:
                     c = abs(float(np.dot(X[:, a], Xr[:, a])))
-                    vec_err = max(vec_err, (1.0 - c) / max(1.0, theta ** 2 / VEC_TOL))
+                    vec_err = max(vec_err, (1.0 - c) / max(1.0, theta ** 2 / vec_tol))
                 else:
                     P = X[:, a:b] @ X[:, a:b].T
                     Pr = Xr[:, a:b] @ Xr[:, a:b].T
                     e = float(np.linalg.norm(P - Pr, 2))
-                    proj_err = max(proj_err, e / max(1.0, theta / PROJ_TOL))
+                    proj_err = max(proj_err, e / max(1.0, theta / proj_tol))
     return Parity(sig, res, orth, vec_err, proj_err, ncl)

@@ -69,6 +69,8 @@ def lib() -> ctypes.CDLL:
     L.wcsvd_batched.restype = I
     L.wcsvd_batched_ex.argtypes = [I, P, P, P, P, P, P, P, D, I, P, ctypes.POINTER(OptsT)]
     L.wcsvd_batched_ex.restype = I
+    L.wcsvd_batched_f32_ex.argtypes = [I, P, P, P, P, P, P, P, ctypes.c_float, I, P, ctypes.POINTER(OptsT)]
+    L.wcsvd_batched_f32_ex.restype = I
     L.wcsvd_workspace_size.argtypes = [I, P, P]
     L.wcsvd_workspace_size.restype = ctypes.c_size_t
     L.wcsvd_status_string.argtypes = [I]
@@ -114,8 +116,9 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
                     max_sweeps: int = 0, stream: int = 0, ldu=None, ldv=None, info_ptr: int = 0,
                     sweeps_inner_ptr: int = 0, workspace_ptr: int = 0, workspace_bytes: int = 0,
                     force_path: int = 0, force_w: int = 0, wcycle_sweeps: int = 0,
-                    inner_sweeps: int = 0) -> None:
-    """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError."""
+                    inner_sweeps: int = 0, fp32: bool = False) -> None:
+    """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError.
+    fp32=True calls wcsvd_batched_f32_ex (float data)."""
     m, n, lda = _arr_i32(m), _arr_i32(n), _arr_i32(lda)
     B = len(m)
     Ap, Sp = _arr_ptr(A_ptrs), _arr_ptr(S_ptrs)
@@ -133,17 +136,18 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
     opts.workspace = workspace_ptr or None
     opts.workspace_bytes = workspace_bytes
     opts.force_path, opts.force_w, opts.wcycle_sweeps, opts.inner_sweeps = force_path, force_w, wcycle_sweeps, inner_sweeps
-    rc = lib().wcsvd_batched_ex(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
-                                Sp.ctypes.data, Up.ctypes.data if Up is not None else None,
-                                Vp.ctypes.data if Vp is not None else None, float(tol), int(max_sweeps),
-                                stream or None, ctypes.byref(opts))
+    fn = lib().wcsvd_batched_f32_ex if fp32 else lib().wcsvd_batched_ex
+    rc = fn(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
+            Sp.ctypes.data, Up.ctypes.data if Up is not None else None,
+            Vp.ctypes.data if Vp is not None else None, float(tol), int(max_sweeps),
+            stream or None, ctypes.byref(opts))
     _check(rc)
 
 
 def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = True,
                 return_info: bool = False, out=None, compute_u: bool | None = None,
                 compute_v: bool | None = None, **kw):
-    """Batched economy SVD of fp64 CUDA tensors on the current stream.
+    """Batched economy SVD of fp64 (or fp32: wcsvd_batched_f32) CUDA tensors on the current stream.
 
     A: tensor [B, m, n] (contiguous) or a sequence of 2-D tensors (sizes may differ).
     Returns (S, U, V) with A = U diag(S) V^T; for a batched tensor S [B, k], U [B, m, k],
@@ -163,53 +167,58 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
         raise WcsvdError(WCSVD_ECUDA, "no CUDA device (this library has no CPU fallback)")
     stream = torch.cuda.current_stream().cuda_stream
     if isinstance(A, torch.Tensor):
-        if A.dim() != 3 or A.dtype != torch.float64 or not A.is_cuda:
-            raise ValueError("A must be a float64 CUDA tensor [B, m, n]")
+        if A.dim() != 3 or A.dtype not in (torch.float64, torch.float32) or not A.is_cuda:
+            raise ValueError("A must be a float64 or float32 CUDA tensor [B, m, n]")
         A = A.contiguous()
         B, m, n = A.shape
         k = min(m, n)
         dev = A.device
+        dt = A.dtype
+        es = A.element_size()
         if out is not None:
             S, Ubuf, Vbuf = out
         else:
-            S = torch.empty(B, k, dtype=torch.float64, device=dev)
-            Ubuf = torch.empty(B, k, m, dtype=torch.float64, device=dev) if cu else None
-            Vbuf = torch.empty(B, k, n, dtype=torch.float64, device=dev) if cv else None
+            S = torch.empty(B, k, dtype=dt, device=dev)
+            Ubuf = torch.empty(B, k, m, dtype=dt, device=dev) if cu else None
+            Vbuf = torch.empty(B, k, n, dtype=dt, device=dev) if cv else None
         info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
         idx = np.arange(B, dtype=np.uint64)
-        a_ptr = A.data_ptr() + idx * np.uint64(8 * m * n)
-        s_ptr = S.data_ptr() + idx * np.uint64(8 * k)
+        a_ptr = A.data_ptr() + idx * np.uint64(es * m * n)
+        s_ptr = S.data_ptr() + idx * np.uint64(es * k)
         # column-major view: the library factors A^T (n x m, lda = n); its "U" (n x k) is our V,
         # its "V" (m x k) is our U.
-        u_ptr = (Vbuf.data_ptr() + idx * np.uint64(8 * k * n)) if Vbuf is not None else None
-        v_ptr = (Ubuf.data_ptr() + idx * np.uint64(8 * k * m)) if Ubuf is not None else None
+        u_ptr = (Vbuf.data_ptr() + idx * np.uint64(es * k * n)) if Vbuf is not None else None
+        v_ptr = (Ubuf.data_ptr() + idx * np.uint64(es * k * m)) if Ubuf is not None else None
         svd_batched_raw(np.full(B, n), np.full(B, m), a_ptr, np.full(B, n), s_ptr, u_ptr, v_ptr,
                         tol=tol, max_sweeps=max_sweeps, stream=stream,
-                        info_ptr=info.data_ptr() if info is not None else 0, **kw)
+                        info_ptr=info.data_ptr() if info is not None else 0, fp32=(es == 4), **kw)
         U = Ubuf.transpose(1, 2) if Ubuf is not None else None
         V = Vbuf.transpose(1, 2) if Vbuf is not None else None
         return (S, U, V, info) if return_info else (S, U, V)
     # list of 2-D tensors
     As = [a.contiguous() for a in A]
     for a in As:
-        if a.dim() != 2 or a.dtype != torch.float64 or not a.is_cuda:
-            raise ValueError("each matrix must be a 2-D float64 CUDA tensor")
+        if a.dim() != 2 or a.dtype not in (torch.float64, torch.float32) or not a.is_cuda:
+            raise ValueError("each matrix must be a 2-D float64 or float32 CUDA tensor")
+    if len({a.dtype for a in As}) > 1:
+        raise ValueError("all matrices of a batch must share one dtype")
     B = len(As)
     if B == 0:
         return ([], [], []) if not return_info else ([], [], [], None)
     dev = As[0].device
+    dt = As[0].dtype
     ms = [a.shape[0] for a in As]
     ns = [a.shape[1] for a in As]
     ks = [min(x, y) for x, y in zip(ms, ns)]
-    Ss = [torch.empty(k, dtype=torch.float64, device=dev) for k in ks]
-    Ub = [torch.empty(k, mm, dtype=torch.float64, device=dev) for k, mm in zip(ks, ms)] if cu else None
-    Vb = [torch.empty(k, nn, dtype=torch.float64, device=dev) for k, nn in zip(ks, ns)] if cv else None
+    Ss = [torch.empty(k, dtype=dt, device=dev) for k in ks]
+    Ub = [torch.empty(k, mm, dtype=dt, device=dev) for k, mm in zip(ks, ms)] if cu else None
+    Vb = [torch.empty(k, nn, dtype=dt, device=dev) for k, nn in zip(ks, ns)] if cv else None
     info = torch.empty(B, dtype=torch.int32, device=dev) if return_info else None
     svd_batched_raw(ns, ms, [a.data_ptr() for a in As], ns, [s.data_ptr() for s in Ss],
                     [v.data_ptr() for v in Vb] if Vb is not None else None,
                     [u.data_ptr() for u in Ub] if Ub is not None else None,
                     tol=tol, max_sweeps=max_sweeps, stream=stream,
-                    info_ptr=info.data_ptr() if info is not None else 0, **kw)
+                    info_ptr=info.data_ptr() if info is not None else 0, fp32=(dt == torch.float32), **kw)
     Us = [u.T for u in Ub] if Ub is not None else None
     Vs = [v.T for v in Vb] if Vb is not None else None
     return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)

@@ -96,37 +96,6 @@ const char* kStatus[] = {"ok", "invalid argument", "not supported", "CUDA error"
 
 using namespace wcsvd;
 
-extern "C" {
-
-const char* wcsvd_version(void) { return "wcsvd 0.1 sm_100a"; }
-
-const char* wcsvd_status_string(int status) {
-  if (status == WCSVD_OK) return kStatus[0];
-  if (status == WCSVD_ENOTSUP) return kStatus[2];
-  if (status == WCSVD_ECUDA) return kStatus[3];
-  if (status == WCSVD_ENOMEM) return kStatus[4];
-  if (status < 0 && status >= -12) return kStatus[1];
-  return "unknown status";
-}
-
-int wcsvd_plan(int m, int n, int force_path, int force_w, wcsvd_plan_t* out) {
-  if (m < 1) return -1;
-  if (n < 1) return -2;
-  if (!out) return -5;
-  if (m > kMaxDim || n > kMaxDim) return WCSVD_ENOTSUP;
-  return plan_one(m, n, force_path, force_w, out);
-}
-
-int wcsvd_round_robin(int np, int step, int* pairs) {
-  if (np < 2 || (np & 1) || step < 0 || step >= np - 1 || !pairs) return -1;
-  for (int k = 0; k < np / 2; ++k) {
-    const int a = rr_content(2 * k, step, np), b = rr_content(2 * k + 1, step, np);
-    pairs[2 * k] = std::min(a, b);
-    pairs[2 * k + 1] = std::max(a, b);
-  }
-  return 0;
-}
-
 static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs, size_t* off_order,
                         size_t* off_status, size_t* off_l1, std::vector<size_t>* l1_off = nullptr,
                         int force_path = 0, int force_w = 0) {
@@ -150,15 +119,12 @@ static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs
   return off;
 }
 
-size_t wcsvd_workspace_size(int batch, const int* m, const int* n) {
-  if (batch <= 0 || !m || !n) return 0;
-  size_t a, b, c, d;
-  return ws_layout(batch, m, n, &a, &b, &c, &d);
-}
-
-int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
-                     double* const* S, double* const* U, double* const* V, double tol,
-                     int max_sweeps, wcsvd_stream_t stream_, const wcsvd_opts* opts) {
+template <typename TI>
+static int batched_impl(int batch, const int* m, const int* n, const TI* const* A, const int* lda,
+                        TI* const* S, TI* const* U, TI* const* V, double tol, int max_sweeps,
+                        wcsvd_stream_t stream_, const wcsvd_opts* opts) {
+  constexpr bool kF32 = sizeof(TI) == 4;
+  const double eps = kF32 ? 5.9604644775390625e-08 : kU53;  // 2^-24 or 2^-53
   cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
   // ---- validation (nothing is enqueued on failure) ----
   if (batch < 0) return -1;
@@ -253,10 +219,12 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     const wcsvd_plan_t& p = plans[b];
     MatDesc& d = h[b];
     std::memset(&d, 0, sizeof(d));
-    d.A = A[b];
-    d.S = S[b];
-    d.U = U ? U[b] : nullptr;
-    d.V = V ? V[b] : nullptr;
+    // typed I/O pointers are carried as double* and reinterpreted by the kernels (d.fp32)
+    d.A = reinterpret_cast<const double*>(A[b]);
+    d.S = reinterpret_cast<double*>(S[b]);
+    d.U = U ? reinterpret_cast<double*>(U[b]) : nullptr;
+    d.V = V ? reinterpret_cast<double*>(V[b]) : nullptr;
+    d.fp32 = kF32 ? 1 : 0;
     d.info = opts ? opts->info : nullptr;
     d.sweeps_inner = opts ? opts->sweeps_inner : nullptr;
     d.m = m[b];
@@ -271,7 +239,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     d.n_pad = p.n_pad;
     d.w = p.w;
     d.w2 = p.w2;
-    d.tol = (tol > 0) ? tol : std::sqrt((double)p.M) * kU53;
+    d.tol = (tol > 0) ? tol : std::sqrt((double)p.M) * eps;
     d.max_sweeps = max_sweeps;
     d.inner_cap = (opts && opts->inner_sweeps > 0) ? opts->inner_sweeps : 1;
     d.inner_cap2 = (opts && opts->wcycle_sweeps > 0) ? opts->wcycle_sweeps : 2;
@@ -317,9 +285,9 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     const int cnt = (int)bk.members.size();
     cudaStream_t st = (nbk > 1) ? side[i] : stream;
     if (bk.path == WCSVD_PATH_L0)
-      e = launch_l0(bk.variant, bk.withv, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
+      e = launch_l0(bk.variant, bk.withv, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
-      e = launch_l1(bk.variant, d_descs, d_order + bucket_off[i], cnt, st);
+      e = launch_l1(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, st);
     if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);
   }
   for (int i = 0; i < (int)side.size(); ++i) {
@@ -330,7 +298,7 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
     if (side[i]) cudaStreamDestroy(side[i]);  // released once its work completes
   }
   if (fork) cudaEventDestroy(fork);
-  if (e == cudaSuccess) e = launch_complete(d_descs, batch, stream);
+  if (e == cudaSuccess) e = launch_complete(kF32 ? 1 : 0, d_descs, batch, stream);
   if (own_ws) cudaFreeAsync(ws, stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -339,10 +307,66 @@ int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const*
   return WCSVD_OK;
 }
 
+
+extern "C" {
+
+const char* wcsvd_version(void) { return "wcsvd 0.1 sm_100a"; }
+
+const char* wcsvd_status_string(int status) {
+  if (status == WCSVD_OK) return kStatus[0];
+  if (status == WCSVD_ENOTSUP) return kStatus[2];
+  if (status == WCSVD_ECUDA) return kStatus[3];
+  if (status == WCSVD_ENOMEM) return kStatus[4];
+  if (status < 0 && status >= -12) return kStatus[1];
+  return "unknown status";
+}
+
+int wcsvd_plan(int m, int n, int force_path, int force_w, wcsvd_plan_t* out) {
+  if (m < 1) return -1;
+  if (n < 1) return -2;
+  if (!out) return -5;
+  if (m > kMaxDim || n > kMaxDim) return WCSVD_ENOTSUP;
+  return plan_one(m, n, force_path, force_w, out);
+}
+
+int wcsvd_round_robin(int np, int step, int* pairs) {
+  if (np < 2 || (np & 1) || step < 0 || step >= np - 1 || !pairs) return -1;
+  for (int k = 0; k < np / 2; ++k) {
+    const int a = rr_content(2 * k, step, np), b = rr_content(2 * k + 1, step, np);
+    pairs[2 * k] = std::min(a, b);
+    pairs[2 * k + 1] = std::max(a, b);
+  }
+  return 0;
+}
+
+size_t wcsvd_workspace_size(int batch, const int* m, const int* n) {
+  if (batch <= 0 || !m || !n) return 0;
+  size_t a, b, c, d;
+  return ws_layout(batch, m, n, &a, &b, &c, &d);
+}
+
+int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                     double* const* S, double* const* U, double* const* V, double tol,
+                     int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts) {
+  return batched_impl<double>(batch, m, n, A, lda, S, U, V, tol, max_sweeps, stream, opts);
+}
+
 int wcsvd_batched(int batch, const int* m, const int* n, const double* const* A, const int* lda,
                   double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
                   wcsvd_stream_t stream) {
-  return wcsvd_batched_ex(batch, m, n, A, lda, S, U, V, tol, max_sweeps, stream, nullptr);
+  return batched_impl<double>(batch, m, n, A, lda, S, U, V, tol, max_sweeps, stream, nullptr);
+}
+
+int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const float* const* A, const int* lda,
+                         float* const* S, float* const* U, float* const* V, float tol, int max_sweeps,
+                         wcsvd_stream_t stream, const wcsvd_opts* opts) {
+  return batched_impl<float>(batch, m, n, A, lda, S, U, V, (double)tol, max_sweeps, stream, opts);
+}
+
+int wcsvd_batched_f32(int batch, const int* m, const int* n, const float* const* A, const int* lda,
+                      float* const* S, float* const* U, float* const* V, float tol, int max_sweeps,
+                      wcsvd_stream_t stream) {
+  return batched_impl<float>(batch, m, n, A, lda, S, U, V, (double)tol, max_sweeps, stream, nullptr);
 }
 
 }  // extern "C"

@@ -66,6 +66,7 @@ struct MatDesc {
   int max_sweeps, inner_cap;
   int inner_cap2;  // W-cycle: cap on Level-2 sweeps per super-pair
   int withv;       // 1: accumulate V_x (requested as V, or as U when swapped); 0: values / U-only mode
+  int fp32;        // 1: A, S, U, V hold float (wcsvd_batched_f32); the pointer fields are reinterpreted
   int idx;      // index of this matrix in the caller's batch (info / status arrays)
   int* status;  // internal per-matrix status flags (workspace), e.g. kNeedsCompletion
 };

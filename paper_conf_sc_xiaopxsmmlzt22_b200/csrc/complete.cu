@@ -30,37 +30,40 @@ __device__ double block_sum(double v, double* red) {
 
 }  // namespace
 
+template <typename TI>
 __global__ void __launch_bounds__(kCT) complete_u_kernel(const MatDesc* __restrict__ descs, int count) {
   const MatDesc d = descs[blockIdx.x];
   if (!d.status || !(d.status[d.idx] & kNeedsCompletion)) return;
-  double* Uw = d.swapped ? d.V : d.U;  // X-space left factor (M x N, ld ldW)
+  TI* Uw = reinterpret_cast<TI*>(d.swapped ? d.V : d.U);  // X-space left factor (M x N, ld ldW)
+  const TI* S = reinterpret_cast<const TI*>(d.S);
   const int ld = d.swapped ? d.ldv : d.ldu;
   if (!Uw) return;
   const int M = d.M, N = d.N;
   __shared__ double x[1024];
   __shared__ double red[kCT / 32];
-  const double thresh = d.S[0] * (double)M * kU53;
+  const double eps = sizeof(TI) == 4 ? 5.9604644775390625e-08 : kU53;
+  const double thresh = (double)S[0] * (double)M * eps;
   int next_e = 0;
   for (int k = 0; k < N; ++k) {
-    if (d.S[k] > thresh) continue;
-    const double sgn = signbit(Uw[(size_t)k * ld]) ? -1.0 : 1.0;  // Z15 flip recorded as -0.0
+    if ((double)S[k] > thresh) continue;
+    const double sgn = signbit((double)Uw[(size_t)k * ld]) ? -1.0 : 1.0;  // Z15 flip recorded as -0.0
     for (;;) {
       for (int r = threadIdx.x; r < M; r += kCT) x[r] = (r == next_e) ? 1.0 : 0.0;
       ++next_e;
       __syncthreads();
       for (int q = 0; q < k; ++q) {
-        const double* uq = Uw + (size_t)q * ld;
+        const TI* uq = Uw + (size_t)q * ld;
         double p = 0.0;
-        for (int r = threadIdx.x; r < M; r += kCT) p = fma(uq[r], x[r], p);
+        for (int r = threadIdx.x; r < M; r += kCT) p = fma((double)uq[r], x[r], p);
         p = block_sum(p, red);
-        for (int r = threadIdx.x; r < M; r += kCT) x[r] = fma(-p, uq[r], x[r]);
+        for (int r = threadIdx.x; r < M; r += kCT) x[r] = fma(-p, (double)uq[r], x[r]);
         __syncthreads();
       }
       double nn = 0.0;
       for (int r = threadIdx.x; r < M; r += kCT) nn = fma(x[r], x[r], nn);
       const double res = sqrt(block_sum(nn, red));
       if (res > 0.5 || next_e >= M) {
-        for (int r = threadIdx.x; r < M; r += kCT) Uw[(size_t)k * ld + r] = sgn * (x[r] / res);
+        for (int r = threadIdx.x; r < M; r += kCT) Uw[(size_t)k * ld + r] = (TI)(sgn * (x[r] / res));
         __syncthreads();
         break;
       }
@@ -69,9 +72,12 @@ __global__ void __launch_bounds__(kCT) complete_u_kernel(const MatDesc* __restri
   (void)count;
 }
 
-cudaError_t launch_complete(const MatDesc* descs, int count, cudaStream_t stream) {
+cudaError_t launch_complete(int fp32, const MatDesc* descs, int count, cudaStream_t stream) {
   if (count <= 0) return cudaSuccess;
-  complete_u_kernel<<<count, kCT, 0, stream>>>(descs, count);
+  if (fp32)
+    complete_u_kernel<float><<<count, kCT, 0, stream>>>(descs, count);
+  else
+    complete_u_kernel<double><<<count, kCT, 0, stream>>>(descs, count);
   return cudaGetLastError();
 }
 

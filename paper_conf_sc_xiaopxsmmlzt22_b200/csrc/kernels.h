@@ -23,13 +23,13 @@ enum L1Variant {
   kL1_32x8 = 13,  // 2w = 32, 8 warps
 };
 
-cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
+cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
 
-cudaError_t launch_l0(int variant, int withv, const MatDesc* descs, const int* order, int count, int maxM,
-                      cudaStream_t stream);
+cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, const int* order, int count,
+                      int maxM, cudaStream_t stream);
 
 }  // namespace wcsvd
 
 namespace wcsvd {
-cudaError_t launch_complete(const MatDesc* descs, int count, cudaStream_t stream);
+cudaError_t launch_complete(int fp32, const MatDesc* descs, int count, cudaStream_t stream);
 }  // namespace wcsvd

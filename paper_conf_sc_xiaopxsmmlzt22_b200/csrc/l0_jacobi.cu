@@ -28,16 +28,36 @@ namespace wcsvd {
 
 namespace {
 
+// Arithmetic type traits: the kernel runs in double (wcsvd_batched) or float (wcsvd_batched_f32).
+template <typename T>
+struct Prec;
+template <>
+struct Prec<double> {
+  using V2 = double2;
+  static constexpr double eps = 1.1102230246251565404e-16;  // 2^-53
+  __device__ static double2 mk(double a, double b) { return make_double2(a, b); }
+  __device__ static double qnan() { return __longlong_as_double(0x7ff8000000000000ULL); }
+};
+template <>
+struct Prec<float> {
+  using V2 = float2;
+  static constexpr float eps = 5.9604644775390625e-08f;  // 2^-24
+  __device__ static float2 mk(float a, float b) { return make_float2(a, b); }
+  __device__ static float qnan() { return __int_as_float(0x7fc00000); }
+};
+
 // Per-CTA state shared by the step functions.
+template <typename T>
 struct L0Ctx {
-  double* part;    // [2 parity][3][RW4][PS]: partial gamma / alpha / beta per (row-thread, pair)
-  double* nrm;     // this warp's [2][NP] cached squared norms per slot (step parity)
-  double2* cs;     // this warp's [G][LP+1] (c, s) per pair (padded against bank conflicts)
+  using V2 = typename Prec<T>::V2;
+  T* part;         // [2 parity][3][RW4][PS]: partial gamma / alpha / beta per (row-thread, pair)
+  T* nrm;          // this warp's [2][NP] cached squared norms per slot (step parity)
+  V2* cs;          // this warp's [G][LP+1] (c, s) per pair (padded against bank conflicts)
   int RW4, PS;
   int lane, g, rt;
   bool isW;
   int dtop, dbot;  // lane k: the slots that the contents of slots 2k, 2k+1 move to
-  double tol2;
+  T tol2;
   int gs;          // global step counter (parity of the partial and norm buffers)
   bool rot_sweep;  // some rotation in the current sweep (identical in every warp)
 };
@@ -46,9 +66,9 @@ struct L0Ctx {
 // slots from x, writes the rotated, moved slots to y. One CTA barrier per step: every warp reduces
 // the row-thread partials itself (lane k = pair k, fixed order) and computes the same rotations,
 // so the (c, s) broadcast needs no second barrier; results are bitwise identical across warps.
-template <int NP, int G, int R, bool FIRST>
-__device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
-                                        double (&y)[R][NP / G]) {
+template <typename T, int NP, int G, int R, bool FIRST>
+__device__ __forceinline__ void l0_step(L0Ctx<T>& cx, const T (&x)[R][NP / G], T (&y)[R][NP / G]) {
+  using V2 = typename Prec<T>::V2;
   constexpr int NL = NP / G;
   constexpr int LP = NL / 2;
   constexpr int NPAIR = NP / 2;
@@ -56,13 +76,13 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
   const int g = cx.g;
   const int par = cx.gs & 1;
   const int SEC = cx.RW4 * cx.PS;  // one partial section
-  double* part = cx.part + par * 3 * SEC;
+  T* part = cx.part + par * 3 * SEC;
   // Phase 1: this thread's partial dot products for its pairs (and squared norms at sweep start).
   if (cx.isW) {
     const int base = cx.rt * cx.PS + g * LP;
 #pragma unroll
     for (int j = 0; j < LP; ++j) {
-      double gm = 0.0, al = 0.0, be = 0.0;
+      T gm = 0, al = 0, be = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         gm = fma(x[r][2 * j], x[r][2 * j + 1], gm);
@@ -85,7 +105,7 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
     const int k = cx.lane;
     if (k < NPAIR) {
       const int PS = cx.PS;
-      double g4[4] = {0.0, 0.0, 0.0, 0.0}, a4[4] = {0.0, 0.0, 0.0, 0.0}, b4[4] = {0.0, 0.0, 0.0, 0.0};
+      T g4[4] = {0, 0, 0, 0}, a4[4] = {0, 0, 0, 0}, b4[4] = {0, 0, 0, 0};
       for (int i = 0; i < cx.RW4; i += 4) {  // rows [RW, RW4) are zero
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -96,8 +116,8 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
           }
         }
       }
-      const double gm = (g4[0] + g4[1]) + (g4[2] + g4[3]);
-      double al, be;
+      const T gm = (g4[0] + g4[1]) + (g4[2] + g4[3]);
+      T al, be;
       if (FIRST) {
         al = (a4[0] + a4[1]) + (a4[2] + a4[3]);
         be = (b4[0] + b4[1]) + (b4[2] + b4[3]);
@@ -105,9 +125,9 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
         al = cx.nrm[par * NP + 2 * k];
         be = cx.nrm[par * NP + 2 * k + 1];
       }
-      double c, sn, t;
+      T c, sn, t;
       rot = jacobi_rotation(al, be, gm, cx.tol2, c, sn, t);
-      cx.cs[(k / LP) * (LP + 1) + (k % LP)] = make_double2(c, sn);
+      cx.cs[(k / LP) * (LP + 1) + (k % LP)] = Prec<T>::mk(c, sn);
       // eq (6) in closed form: alpha' = alpha + t gamma, beta' = beta - t gamma
       cx.nrm[(par ^ 1) * NP + cx.dtop] = rot ? fma(t, gm, al) : al;
       cx.nrm[(par ^ 1) * NP + cx.dbot] = rot ? fma(-t, gm, be) : be;
@@ -119,17 +139,17 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
   // Outputs of local pair j: top -> top[j+1], bot -> bot[j-1]. Group 0 keeps top[0] and sends
   // bot[0] to its top[1]; other groups receive top[0] from the left neighbour lane; the last group
   // moves its last top to its last bot, the others receive their last bot from the right.
-  double top0[R], send_l[R], send_r[R];
-  const double2* cs = cx.cs + g * (LP + 1);
+  T top0[R], send_l[R], send_r[R];
+  const V2* cs = cx.cs + g * (LP + 1);
 #pragma unroll
   for (int j = 0; j < LP; ++j) {
-    const double2 p = cs[j];
+    const V2 p = cs[j];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      const double a = x[r][2 * j], b = x[r][2 * j + 1];
+      const T a = x[r][2 * j], b = x[r][2 * j + 1];
       // eq (3): (a^_i, a^_j) = (a_i, a_j) [[c, -s], [s, c]]
-      const double na = fma(p.y, b, p.x * a);
-      const double nb = fma(-p.y, a, p.x * b);
+      const T na = fma(p.y, b, p.x * a);
+      const T nb = fma(-p.y, a, p.x * b);
       if (j == 0) top0[r] = na;
       else if (j + 1 < LP) y[r][2 * (j + 1)] = na;
       else send_r[r] = na;
@@ -140,7 +160,7 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
   const bool gfirst = (g == 0), glast = (g == G - 1);
 #pragma unroll
   for (int r = 0; r < R; ++r) {
-    double from_left = 0.0, from_right = 0.0;
+    T from_left = 0, from_right = 0;
     if (G > 1) {
       from_left = __shfl_up_sync(0xffffffffu, send_r[r], 1);
       from_right = __shfl_down_sync(0xffffffffu, send_l[r], 1);
@@ -153,37 +173,39 @@ __device__ __forceinline__ void l0_step(L0Ctx& cx, const double (&x)[R][NP / G],
 }
 
 // One sweep of NP-1 steps starting in x; ends in y with every slot back in its original column.
-template <int NP, int G, int R>
-__device__ __forceinline__ void l0_sweep(L0Ctx& cx, double (&x)[R][NP / G], double (&y)[R][NP / G]) {
+template <typename T, int NP, int G, int R>
+__device__ __forceinline__ void l0_sweep(L0Ctx<T>& cx, T (&x)[R][NP / G], T (&y)[R][NP / G]) {
   cx.rot_sweep = false;
-  l0_step<NP, G, R, true>(cx, x, y);
+  l0_step<T, NP, G, R, true>(cx, x, y);
   for (int i = 0; i < (NP - 2) / 2; ++i) {
-    l0_step<NP, G, R, false>(cx, y, x);
-    l0_step<NP, G, R, false>(cx, x, y);
+    l0_step<T, NP, G, R, false>(cx, y, x);
+    l0_step<T, NP, G, R, false>(cx, x, y);
   }
 }
 
 }  // namespace
 
 // Shared-memory bytes of one CTA (must match the carve-up in the kernel).
-template <int NP, int G, int R, bool WITHV>
+template <typename T, int NP, int G, int R, bool WITHV>
 size_t l0_smem_bytes(int M, int threads) {
   const int RW4 = ((M + R - 1) / R + 3) / 4 * 4;
   const int PS = NP / 2 + 1;
   const int RV = WITHV ? NP / R : RW4;  // rows of the sign-rule scratch (V rows, or X rows)
   const int LP = NP / G / 2;
   const int NW = threads / 32;
-  return sizeof(double) * 6 * (size_t)RW4 * PS                         // partials, 2 parities
-         + (size_t)NW * (sizeof(double2) * G * (LP + 1) + sizeof(double) * 2 * NP)  // per-warp cs, nrm
-         + sizeof(double) * (2 * NP + (size_t)RV * NP) + sizeof(int) * (NP + 8);
+  return sizeof(T) * 6 * (size_t)RW4 * PS                              // partials, 2 parities
+         + (size_t)NW * (2 * sizeof(T) * G * (LP + 1) + sizeof(T) * 2 * NP)  // per-warp cs, nrm
+         + sizeof(T) * (2 * NP + (size_t)RV * NP) + sizeof(int) * (NP + 8) + 16;
 }
 
 // One CTA per matrix. Thread t: group g = t % G, row-thread rt = t / G. Row-threads [0, RW) hold
 // rows rt*R .. rt*R+R-1 of X; row-threads [RW, RW+RV) hold rows of V (RV = NP/R); the rest (to a
 // multiple of 32) hold zeros and only take part in shuffles.
-template <int NP, int G, int R, int MAXT, bool WITHV>
+template <typename T, int NP, int G, int R, int MAXT, bool WITHV>
 __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restrict__ descs,
                                                         const int* __restrict__ order) {
+  // T: arithmetic and I/O type (double for wcsvd_batched, float for wcsvd_batched_f32).
+  using V2 = typename Prec<T>::V2;
   constexpr int NL = NP / G;
   constexpr int LP = NL / 2;
   constexpr int NPAIR = NP / 2;
@@ -192,7 +214,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   const int M = d.M, N = d.N;
   const int RW = (M + R - 1) / R;
   const int PS = NPAIR + 1;  // odd stride (doubles): conflict-free partial writes and reads
-  const int T = blockDim.x;
+  const int NT = blockDim.x;
   const int tid = threadIdx.x;
   const int g = tid % G;
   const int rt = tid / G;
@@ -201,47 +223,48 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
 
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int RW4 = (RW + 3) / 4 * 4;  // partial rows padded to 4 (zeros)
-  const int NWARP = T / 32;
-  double* s_part = reinterpret_cast<double*>(smem_raw);                   // [2][3][RW4][PS]
-  double2* s_csw = reinterpret_cast<double2*>(s_part + 6 * RW4 * PS);     // [NWARP][G][LP+1]
-  double* s_nrmw = reinterpret_cast<double*>(s_csw + NWARP * G * (LP + 1));  // [NWARP][2][NP]
-  double* s_sig = s_nrmw + NWARP * 2 * NP;                                // [NP]
-  double* s_sgn = s_sig + NP;                                             // [NP]
+  const int NWARP = NT / 32;
+  unsigned long long* s_max = reinterpret_cast<unsigned long long*>(smem_raw);  // [2] (16 B)
+  T* s_part = reinterpret_cast<T*>(smem_raw + 16);                        // [2][3][RW4][PS]
+  V2* s_csw = reinterpret_cast<V2*>(s_part + 6 * RW4 * PS);               // [NWARP][G][LP+1]
+  T* s_nrmw = reinterpret_cast<T*>(s_csw + NWARP * G * (LP + 1));         // [NWARP][2][NP]
+  T* s_sig = s_nrmw + NWARP * 2 * NP;                                     // [NP]
+  T* s_sgn = s_sig + NP;                                                  // [NP]
   const int SR = WITHV ? RV : RW4;                                        // sign-rule rows
-  double* s_vbest = s_sgn + NP;                                           // [SR][NP]
+  T* s_vbest = s_sgn + NP;                                                // [SR][NP]
   int* s_rank = reinterpret_cast<int*>(s_vbest + SR * NP);                // [NP]
   int* s_flags = s_rank + NP;                                             // [8]
-  unsigned long long* s_max = reinterpret_cast<unsigned long long*>(s_flags + 4);
   if (tid < 4) s_flags[tid] = 0;
   if (tid == 0) *s_max = 0ull;
-  for (int e = tid; e < 6 * RW4 * PS; e += T) s_part[e] = 0.0;
+  for (int e = tid; e < 6 * RW4 * PS; e += NT) s_part[e] = T(0);
   __syncthreads();
 
   // ---- Stage-in: X = A (m >= n) or A^T (m < n), zero-padded; V = I. ----
-  double xa[R][NL], xb[R][NL];
+  T xa[R][NL], xb[R][NL];
   bool bad = false;
-  double amax = 0.0;
+  T amax = 0;
+  const T* Ain = reinterpret_cast<const T*>(d.A);
 #pragma unroll
   for (int r = 0; r < R; ++r) {
 #pragma unroll
     for (int l = 0; l < NL; ++l) {
       const int col = g * NL + l;
-      double v = 0.0;
+      T v = 0;
       if (isW) {
         const int row = rt * R + r;
         if (row < M && col < N) {
-          v = d.swapped ? d.A[(size_t)row * d.lda + col] : d.A[(size_t)col * d.lda + row];
+          v = d.swapped ? Ain[(size_t)row * d.lda + col] : Ain[(size_t)col * d.lda + row];
           bad |= !isfinite(v);
           amax = fmax(amax, fabs(v));
         }
       } else if (isV) {
-        v = ((rt - RW) * R + r == col) ? 1.0 : 0.0;
+        v = ((rt - RW) * R + r == col) ? T(1) : T(0);
       }
       xa[r][l] = v;
     }
   }
   if (bad) atomicOr(&s_flags[2], 1);
-  if (isW && amax > 0.0) atomicMax(s_max, (unsigned long long)__double_as_longlong(amax));
+  if (isW && amax > T(0)) atomicMax(s_max, (unsigned long long)__double_as_longlong((double)amax));
   __syncthreads();
   const bool nonfinite = s_flags[2] != 0;
   // Exact power-of-two pre-scaling to max|x| in [0.5, 1): every product in the iteration stays in
@@ -251,7 +274,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   if (!nonfinite && *s_max != 0ull) {
     frexp(__longlong_as_double((long long)*s_max), &sexp);
     if (isW) {
-      const double f = ldexp(1.0, -sexp);
+      const T f = (T)ldexp(1.0, -sexp);
 #pragma unroll
       for (int r = 0; r < R; ++r)
 #pragma unroll
@@ -260,7 +283,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   }
 
   const int lane = tid & 31, warp = tid >> 5;
-  L0Ctx cx;
+  L0Ctx<T> cx;
   cx.part = s_part;
   cx.nrm = s_nrmw + warp * 2 * NP;
   cx.cs = s_csw + warp * G * (LP + 1);
@@ -272,7 +295,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   cx.isW = isW;
   cx.dtop = rr_dest(2 * lane, NP);
   cx.dbot = rr_dest(2 * lane + 1, NP);
-  cx.tol2 = d.tol * d.tol;
+  cx.tol2 = (T)(d.tol * d.tol);
   cx.gs = 0;
   cx.rot_sweep = false;
   int sweep = 0;
@@ -280,11 +303,11 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   bool in_b = false;
   if (!nonfinite) {
     for (;;) {
-      l0_sweep<NP, G, R>(cx, xa, xb);  // ends in xb
+      l0_sweep<T, NP, G, R>(cx, xa, xb);  // ends in xb
       ++sweep;
       if (!cx.rot_sweep) { converged = true; in_b = true; break; }
       if (sweep >= d.max_sweeps) { in_b = true; break; }
-      l0_sweep<NP, G, R>(cx, xb, xa);  // ends in xa
+      l0_sweep<T, NP, G, R>(cx, xb, xa);  // ends in xa
       ++sweep;
       if (!cx.rot_sweep) { converged = true; break; }
       if (sweep >= d.max_sweeps) break;
@@ -303,7 +326,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   if (isW) {
 #pragma unroll
     for (int l = 0; l < NL; ++l) {
-      double a = 0.0;
+      T a = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r) a = fma(xa[r][l], xa[r][l], a);
       const int col = g * NL + l;  // [RW][NP] view over the first two partial sections
@@ -315,7 +338,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
   if (WITHV ? isV : isW) {
 #pragma unroll
     for (int l = 0; l < NL; ++l) {
-      double best = 0.0;
+      T best = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r)
         if (fabs(xa[r][l]) > fabs(best)) best = xa[r][l];
@@ -323,45 +346,45 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
     }
   }
   __syncthreads();
-  for (int j = tid; j < NP; j += T) {
+  for (int j = tid; j < NP; j += NT) {
     const int base = (j < NPAIR ? 0 : RW4) * PS + (j % NPAIR);
-    double a4[4] = {0.0, 0.0, 0.0, 0.0};
+    T a4[4] = {0, 0, 0, 0};
     for (int i = 0; i < RW; i += 4) {
 #pragma unroll
       for (int u = 0; u < 4; ++u) a4[u] += s_part[base + (i + u) * PS];
     }
     s_sig[j] = sqrt((a4[0] + a4[1]) + (a4[2] + a4[3]));  // of the pre-scaled X
-    double best = 0.0;
+    T best = 0;
     for (int i = 0; i < (WITHV ? RV : RW); ++i) {
-      const double v = s_vbest[i * NP + j];
+      const T v = s_vbest[i * NP + j];
       if (fabs(v) > fabs(best)) best = v;
     }
-    s_sgn[j] = (best < 0.0) ? -1.0 : 1.0;
+    s_sgn[j] = (best < T(0)) ? T(-1) : T(1);
   }
   __syncthreads();
-  for (int j = tid; j < NP; j += T) {
+  for (int j = tid; j < NP; j += NT) {
     int rk = -1;
     if (j < N && nonfinite) {
       rk = j;  // NaN sigmas: identity order, every column written
     } else if (j < N) {
       rk = 0;
-      const double sj = s_sig[j];
+      const T sj = s_sig[j];
       for (int i = 0; i < N; ++i) {
-        const double si = s_sig[i];
+        const T si = s_sig[i];
         rk += (si > sj) || (si == sj && i < j);
       }
     }
     s_rank[j] = rk;
   }
   __syncthreads();
-  double sig1 = 0.0;
+  T sig1 = 0;
   for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
-  const double thresh = sig1 * (double)M * kU53;  // Z14 rank threshold (scale-invariant)
-  const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
+  const T thresh = sig1 * (T)M * Prec<T>::eps;  // Z14 rank threshold (scale-invariant)
+  const T nanv = Prec<T>::qnan();
   // X-space factors: U_w -> U (V if swapped), V_x -> V (U if swapped).
-  double* dstW = d.swapped ? d.V : d.U;
+  T* dstW = reinterpret_cast<T*>(d.swapped ? d.V : d.U);
   const int ldW = d.swapped ? d.ldv : d.ldu;
-  double* dstV = d.swapped ? d.U : d.V;
+  T* dstV = reinterpret_cast<T*>(d.swapped ? d.U : d.V);
   const int ldV = d.swapped ? d.ldu : d.ldv;
   bool needs_completion = false;
   if (isW && dstW) {
@@ -370,15 +393,15 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
       const int col = g * NL + l;
       if (col < N) {
         const int rk = s_rank[col];
-        const double sj = s_sig[col];
-        const double sgn = s_sgn[col];
+        const T sj = s_sig[col];
+        const T sgn = s_sgn[col];
         const bool ok = sj > thresh;
         needs_completion |= !ok;
 #pragma unroll
         for (int r = 0; r < R; ++r) {
           const int row = rt * R + r;
           if (row < M)  // rank-deficient columns: signed zero, completed by complete_u_kernel
-            dstW[(size_t)rk * ldW + row] = nonfinite ? nanv : (ok ? sgn * (xa[r][l] / sj) : sgn * 0.0);
+            dstW[(size_t)rk * ldW + row] = nonfinite ? nanv : (ok ? sgn * (xa[r][l] / sj) : sgn * T(0));
         }
       }
     }
@@ -389,7 +412,7 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
       const int col = g * NL + l;
       if (col < N) {
         const int rk = s_rank[col];
-        const double sgn = s_sgn[col];
+        const T sgn = s_sgn[col];
 #pragma unroll
         for (int r = 0; r < R; ++r) {
           const int vrow = (rt - RW) * R + r;
@@ -399,7 +422,8 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
     }
   }
   if (needs_completion && !nonfinite) atomicOr(&s_flags[3], 1);
-  for (int j = tid; j < N; j += T) d.S[s_rank[j]] = nonfinite ? nanv : ldexp(s_sig[j], sexp);
+  T* Sout = reinterpret_cast<T*>(d.S);
+  for (int j = tid; j < N; j += NT) Sout[s_rank[j]] = nonfinite ? nanv : (T)ldexp((double)s_sig[j], sexp);
   __syncthreads();
   if (tid == 0) {
     if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
@@ -409,41 +433,45 @@ __global__ void __launch_bounds__(MAXT) l0_jacobi_kernel(const MatDesc* __restri
 }
 
 // ---- launcher ----
-template <int NP, int G, int R, int MAXT, bool WITHV>
+template <typename T, int NP, int G, int R, int MAXT, bool WITHV>
 static cudaError_t launch_l0_t(const MatDesc* descs, const int* order, int count, int maxM,
                                cudaStream_t stream) {
   const int RW = (maxM + R - 1) / R;
   int threads = (RW + (WITHV ? NP / R : 0)) * G;
   threads = (threads + 31) / 32 * 32;
   if (threads > MAXT) return cudaErrorInvalidConfiguration;
-  const size_t smem = l0_smem_bytes<NP, G, R, WITHV>(maxM, threads);
-  auto kern = l0_jacobi_kernel<NP, G, R, MAXT, WITHV>;
+  const size_t smem = l0_smem_bytes<T, NP, G, R, WITHV>(maxM, threads);
+  auto kern = l0_jacobi_kernel<T, NP, G, R, MAXT, WITHV>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<count, threads, smem, stream>>>(descs, order);
   return cudaGetLastError();
 }
 
-template <bool WITHV>
+template <typename T, bool WITHV>
 static cudaError_t launch_l0_v(int variant, const MatDesc* descs, const int* order, int count, int maxM,
                                cudaStream_t stream) {
   switch (variant) {
-    case kL0_8:   return launch_l0_t<8, 1, 8, 256, WITHV>(descs, order, count, maxM, stream);
-    case kL0_16:  return launch_l0_t<16, 2, 8, 256, WITHV>(descs, order, count, maxM, stream);
-    case kL0_32:  return launch_l0_t<32, 2, 4, 256, WITHV>(descs, order, count, maxM, stream);
-    case kL0_32s: return launch_l0_t<32, 2, 1, 512, WITHV>(descs, order, count, maxM, stream);
-    case kL0_48:  return launch_l0_t<48, 2, 2, 256, WITHV>(descs, order, count, maxM, stream);
-    case kL0_64:  return launch_l0_t<64, 8, 8, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_8:   return launch_l0_t<T, 8, 1, 8, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_16:  return launch_l0_t<T, 16, 2, 8, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_32:  return launch_l0_t<T, 32, 2, 4, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_32s: return launch_l0_t<T, 32, 2, 1, 512, WITHV>(descs, order, count, maxM, stream);
+    case kL0_48:  return launch_l0_t<T, 48, 2, 2, 256, WITHV>(descs, order, count, maxM, stream);
+    case kL0_64:  return launch_l0_t<T, 64, 8, 8, 256, WITHV>(descs, order, count, maxM, stream);
     default: return cudaErrorInvalidValue;
   }
 }
 
-// Variant table (planner ids). E = R * NP / G doubles per thread. withv = 0: V_x is not accumulated
+// Variant table (planner ids). E = R * NP / G elements per thread. withv = 0: V_x is not accumulated
 // (it is not requested; §8(f4) values / U-only mode) -- half the threads and registers per matrix.
-cudaError_t launch_l0(int variant, int withv, const MatDesc* descs, const int* order, int count, int maxM,
-                      cudaStream_t stream) {
-  return withv ? launch_l0_v<true>(variant, descs, order, count, maxM, stream)
-               : launch_l0_v<false>(variant, descs, order, count, maxM, stream);
+// fp32 = 1: the fp32 variant (§8(f1)), iterated in float.
+cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, const int* order, int count,
+                      int maxM, cudaStream_t stream) {
+  if (fp32)
+    return withv ? launch_l0_v<float, true>(variant, descs, order, count, maxM, stream)
+                 : launch_l0_v<float, false>(variant, descs, order, count, maxM, stream);
+  return withv ? launch_l0_v<double, true>(variant, descs, order, count, maxM, stream)
+               : launch_l0_v<double, false>(variant, descs, order, count, maxM, stream);
 }
 
 }  // namespace wcsvd

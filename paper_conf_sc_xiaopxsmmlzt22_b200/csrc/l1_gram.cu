@@ -535,9 +535,11 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, cons
 
 }  // namespace
 
-template <int W2, int NW>
+template <int W2, int NW, typename TI>
 __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
                                                              const int* __restrict__ order) {
+  // TI: type of A, S, U, V in the caller's memory (double, or float for wcsvd_batched_f32); the
+  // iteration always runs on the fp64 working copy.
   using C = PairCfg<W2>;
   const MatDesc d = descs[order[blockIdx.x]];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -580,7 +582,8 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     const int c = (int)(e / mp), r = (int)(e % mp);
     double v = 0.0;
     if (r < M && c < N) {
-      v = d.swapped ? d.A[(size_t)r * d.lda + c] : d.A[(size_t)c * d.lda + r];
+      const TI* Ain = reinterpret_cast<const TI*>(d.A);
+      v = (double)(d.swapped ? Ain[(size_t)r * d.lda + c] : Ain[(size_t)c * d.lda + r]);
       bad |= !isfinite(v);
       amax = fmax(amax, fabs(v));
     }
@@ -749,9 +752,9 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
   const double thresh = sig1 * (double)M * kU53;
   const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
-  double* dstW = d.swapped ? d.V : d.U;
+  TI* dstW = reinterpret_cast<TI*>(d.swapped ? d.V : d.U);
   const int ldW = d.swapped ? d.ldv : d.ldu;
-  double* dstV = d.swapped ? d.U : d.V;
+  TI* dstV = reinterpret_cast<TI*>(d.swapped ? d.U : d.V);
   const int ldV = d.swapped ? d.ldu : d.ldv;
   bool needs_completion = false;
   for (int j = warp; j < N; j += NW) {
@@ -762,13 +765,13 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     if (dstW) {
       const double* col = Wm + (size_t)j * mp;
       for (int r = lane; r < M; r += 32)
-        dstW[(size_t)rk * ldW + r] = nonfinite ? nanv : (ok ? sgn * (col[r] / sj) : sgn * 0.0);
+        dstW[(size_t)rk * ldW + r] = (TI)(nonfinite ? nanv : (ok ? sgn * (col[r] / sj) : sgn * 0.0));
     }
     if (dstV) {
       const double* vc = Vm + (size_t)j * np;
-      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = nonfinite ? nanv : sgn * vc[i];
+      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = (TI)(nonfinite ? nanv : sgn * vc[i]);
     }
-    if (lane == 0) d.S[rk] = nonfinite ? sj : ldexp(sj, sexp);
+    if (lane == 0) reinterpret_cast<TI*>(d.S)[rk] = (TI)(nonfinite ? sj : ldexp(sj, sexp));
   }
   if (needs_completion && !nonfinite && lane == 0) atomicOr(&s_flags[3], 1);
   __syncthreads();
@@ -781,25 +784,31 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
 }
 
-template <int W2, int NW>
+template <int W2, int NW, typename TI>
 static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
   size_t smem = NW * WarpSmem<W2>::bytes();
   const size_t fin = 3 * 8 * 1024;  // finalisation arrays alias the warp buffers
   if (smem < fin) smem = fin;
-  auto kern = l1_gram_kernel<W2, NW>;
+  auto kern = l1_gram_kernel<W2, NW, TI>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<count, NW * 32, smem, stream>>>(descs, order);
   return cudaGetLastError();
 }
 
-cudaError_t launch_l1(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
+template <typename TI>
+static cudaError_t launch_l1_v(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
   switch (variant) {
-    case kL1_16x4: return launch_l1_t<16, 4>(descs, order, count, stream);
-    case kL1_32x4: return launch_l1_t<32, 4>(descs, order, count, stream);
-    case kL1_32x8: return launch_l1_t<32, 8>(descs, order, count, stream);
+    case kL1_16x4: return launch_l1_t<16, 4, TI>(descs, order, count, stream);
+    case kL1_32x4: return launch_l1_t<32, 4, TI>(descs, order, count, stream);
+    case kL1_32x8: return launch_l1_t<32, 8, TI>(descs, order, count, stream);
     default: return cudaErrorInvalidValue;
   }
+}
+
+cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
+  return fp32 ? launch_l1_v<float>(variant, descs, order, count, stream)
+              : launch_l1_v<double>(variant, descs, order, count, stream);
 }
 
 }  // namespace wcsvd

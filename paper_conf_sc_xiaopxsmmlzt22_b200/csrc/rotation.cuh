@@ -35,6 +35,27 @@ __device__ __forceinline__ bool jacobi_rotation(double alpha, double beta, doubl
   return true;
 }
 
+// fp32 variant of the same evaluation (wcsvd_batched_f32, Level 0).
+__device__ __forceinline__ bool jacobi_rotation(float alpha, float beta, float gamma, float tol2, float& c,
+                                                float& s, float& t) {
+  c = 1.0f;
+  s = 0.0f;
+  t = 0.0f;
+  const float ab = alpha * beta;
+  const float g2 = gamma * gamma;
+  if (!(ab > 0.0f) || g2 <= tol2 * ab) return false;
+  const float d = alpha - beta, ad = fabsf(d);
+  const float r = sqrtf(fmaf(d, d, 4.0f * g2));
+  const float rp = r + ad;
+  const float q = rsqrtf(2.0f * r * rp);
+  const float sg = (d == 0.0f || ((d > 0.0f) == (gamma > 0.0f))) ? 2.0f : -2.0f;
+  const float sq = sg * fabsf(gamma) * q;
+  c = rp * q;
+  s = sq;
+  t = 2.0f * r * sq * q;
+  return true;
+}
+
 // Same rotation with the angle evaluated in fp32 (R-ROT32). The threshold test and d
 // are fp64; (d, gamma) are rescaled by an exact power of two into fp32 range (t is homogeneous of
 // degree 0 in them), t is formed in fp32 (~1e-7 relative), then c = 1/sqrt(1 + t^2) and s = t c are
