@@ -61,9 +61,6 @@ struct PairCfg {
   static constexpr int CG = W2 / 8;         // 8-column groups per pair panel
   static constexpr int NTU = CG * (CG + 1) / 2;  // upper tiles of the 2w x 2w Gram
   static constexpr int BS = W2 + 1;         // SMEM row stride of 2w x 2w buffers (doubles)
-  static constexpr int NPR = W2 / 2;        // rotation pairs per EVD step
-  static constexpr int NQ = NPR * (NPR - 1) / 2;  // off-diagonal quads (k < l) per EVD step
-  static constexpr int QPL = (NQ + 31) / 32;       // quads per lane
   static_assert(W2 == 16 || W2 == 32, "pair panel width");
 };
 
@@ -324,132 +321,176 @@ __device__ __forceinline__ void apply_rotation(double* base, int ld, int rows, i
   }
 }
 
-// Off-diagonal quads (k < l) of an EVD step handled by this lane: q = lane + 32 i.
+// ---- Inner EVD storage: B in "slot" order, moved along with the round-robin ring ----
+// B (symmetric, 2w x 2w) is kept as its upper triangle indexed by *slot*: the pair k of every step
+// is always slots (2k, 2k+1), so the elements a lane reads (its 2x2 quads) sit at the same
+// addresses at every step; the rotated values are written straight to the slots their rows and
+// columns move to (common.cuh rr_dest), into a second buffer (ping-pong). After 2w-1 steps every
+// index is back in its own slot. Element (a, b), a <= b, lives at a*W2 + (b ^ ((a >> 1) & (w-1))):
+// the XOR swizzle spreads each step's 32 lanes over the shared-memory banks (the two elements of a
+// quad row stay one aligned 16-byte pair, loaded as one double2).
 template <int W2>
-struct QuadMap {
-  int k[PairCfg<W2>::QPL], l[PairCfg<W2>::QPL];
+__host__ __device__ __forceinline__ int evd_phys(int a, int b) {
+  return a * W2 + (b ^ ((a >> 1) & (W2 / 2 - 1)));
+}
+template <int W2>
+__device__ __forceinline__ int evd_phys_sym(int a, int b) {
+  return (a <= b) ? evd_phys<W2>(a, b) : evd_phys<W2>(b, a);
+}
+
+// Lane-static EVD work map. Lane L works for pair k = L mod (w) (it evaluates that pair's rotation,
+// redundantly with the other lanes of the same k) and owns the off-diagonal quads {k, (k+d) mod w}
+// for its share of d = 1 .. w/2 (d = w/2 only from the lower k, so every unordered pair of pairs is
+// owned exactly once). Offsets are element offsets into a buffer.
+template <int W2>
+struct EvdMap {
+  static constexpr int NPR = W2 / 2, LPP = 32 / NPR, HALF = NPR / 2;
+  static constexpr int QPL = (HALF + LPP - 1) / LPP;  // quads per lane
+  int q[QPL];       // bits 0-10 load offset (row 2lo, aligned column pair), 11 swap, 12 own-is-lo,
+                    // 13 valid, 16-19 partner pair
+  int st[QPL][2];   // store offsets of e00 | e01 << 16 and e10 | e11 << 16
+  int dld01, dld2;  // diagonal block loads: (2k,2k) | (2k+1,2k+1) << 16, (2k,2k+1)
+  int dst01, dst2;  // diagonal block stores (moved slots)
   __device__ __forceinline__ void init(int lane) {
-    constexpr int NPR = PairCfg<W2>::NPR, NQ = PairCfg<W2>::NQ;
+    const int k = lane & (NPR - 1), h = lane / NPR;
 #pragma unroll
-    for (int i = 0; i < PairCfg<W2>::QPL; ++i) {
-      int q = lane + 32 * i, kk = 0;
-      k[i] = -1;
-      l[i] = -1;
-      if (q < NQ) {
-        while (q >= NPR - 1 - kk) { q -= NPR - 1 - kk; ++kk; }
-        k[i] = kk;
-        l[i] = kk + 1 + q;
-      }
+    for (int i = 0; i < QPL; ++i) {
+      const int d = 1 + h * QPL + i;
+      const bool valid = d < HALF || (d == HALF && k < HALF);
+      const int l = (k + d) & (NPR - 1), lo = min(k, l), hi = max(k, l);
+      q[i] = 0;
+      st[i][0] = st[i][1] = 0;
+      if (!valid) continue;
+      q[i] = (2 * lo * W2 + ((2 * hi) ^ (lo & ~1))) | ((lo & 1) << 11) | ((k < l) << 12) | (1 << 13) | (l << 16);
+      int o[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) o[e] = evd_phys_sym<W2>(rr_dest(2 * lo + (e >> 1), W2), rr_dest(2 * hi + (e & 1), W2));
+      st[i][0] = o[0] | (o[1] << 16);
+      st[i][1] = o[2] | (o[3] << 16);
     }
+    dld01 = evd_phys<W2>(2 * k, 2 * k) | (evd_phys<W2>(2 * k + 1, 2 * k + 1) << 16);
+    dld2 = evd_phys<W2>(2 * k, 2 * k + 1);
+    const int a0 = rr_dest(2 * k, W2), a1 = rr_dest(2 * k + 1, W2);
+    dst01 = evd_phys<W2>(a0, a0) | (evd_phys<W2>(a1, a1) << 16);
+    dst2 = evd_phys_sym<W2>(a0, a1);
   }
 };
 
-// One inner EVD step r (round-robin over 2w indices): lanes k < w compute the
-// rotations of the step's disjoint pairs (p_k, q_k) and apply the annihilating 2x2 update to their
-// own diagonal quad; then every off-diagonal quad (k < l) of B' = G^T B G is updated from 4 loads
-// and written with its mirror (B symmetric); J <- J G in slot order. rr[k] holds
-// (p BS, q BS, p, q) of pair k at this step (precomputed round-robin table). A step in which no pair
-// rotates only moves J's slots.
+// One inner EVD step (round-robin over 2w indices): every lane evaluates the rotation
+// of its pair k = (slots 2k, 2k+1) from the diagonal block; lanes k < w publish (c, s) and write the
+// annihilated diagonal block (eq 6 analogue, exact zero off-diagonal); every off-diagonal quad of
+// B' = G^T B G is updated from one load per quad row and written, like the
+// diagonal blocks, to the slots its indices move to in Bn; J <- J G in slot order (x -> y rename).
+// A step in which no pair rotates only moves B and J.
 template <int W2>
-__device__ __forceinline__ bool evd_step(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int2* __restrict__ rr,
-                                         int lane, double tol2, const double (&x)[W2], double (&y)[W2]) {
-  using C = PairCfg<W2>;
-  constexpr int NPR = C::NPR, QPL = C::QPL, BS = C::BS;
-  double* B = ws.B;
-  // Off-diagonal quad elements are written only by their owner lane, so they are loaded before the
-  // rotation chain of the parameter lanes and their latency overlaps it.
-  int ak[QPL], al[QPL];  // packed (p, q) of quads' row pair k and column pair l: p | q << 16
+__device__ __forceinline__ bool evd_step(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
+                                         const EvdMap<W2>& em, int lane, double tol2, const double (&x)[W2],
+                                         double (&y)[W2]) {
+  constexpr int NPR = W2 / 2, QPL = EvdMap<W2>::QPL;
+  const double bpp = Bc[em.dld01 & 0xffff], bqq = Bc[em.dld01 >> 16], bpq = Bc[em.dld2];
+  double c, s, t;
+  const bool rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
+  if (lane < NPR) {
+    cs[lane] = make_double2(c, s);
+    Bn[em.dst01 & 0xffff] = rot ? fma(t, bpq, bpp) : bpp;
+    Bn[em.dst01 >> 16] = rot ? fma(-t, bpq, bqq) : bqq;
+    Bn[em.dst2] = rot ? 0.0 : bpq;
+  }
   double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
 #pragma unroll
   for (int i = 0; i < QPL; ++i) {
-    if (qm.k[i] >= 0) {
-      const int2 xk = rr[qm.k[i]], xl = rr[qm.l[i]];
-      ak[i] = xk.x | (xk.y << 16);
-      al[i] = xl.x | (xl.y << 16);
-      b00[i] = B[xk.x * BS + xl.x];
-      b01[i] = B[xk.x * BS + xl.y];
-      b10[i] = B[xk.y * BS + xl.x];
-      b11[i] = B[xk.y * BS + xl.y];
-    }
-  }
-  bool rot = false;
-  if (lane < NPR) {
-    const int2 pq = rr[lane];
-    const int pp = pq.x * BS + pq.x, qq = pq.y * BS + pq.y, pqo = pq.x * BS + pq.y, qpo = pq.y * BS + pq.x;
-    const double bpp = B[pp], bqq = B[qq], bpq = B[pqo];
-    double c, s, t;
-    rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
-    ws.cs[lane] = make_double2(c, s);
-    if (rot) {  // annihilated pair: closed-form diagonal (eq 6 analogue), exact zero off-diagonal
-      B[pp] = fma(t, bpq, bpp);
-      B[qq] = fma(-t, bpq, bqq);
-      B[pqo] = 0.0;
-      B[qpo] = 0.0;
+    if (em.q[i] & (1 << 13)) {
+      const int o = em.q[i] & 0x7ff;
+      const double2 v0 = *reinterpret_cast<const double2*>(Bc + o);
+      const double2 v1 = *reinterpret_cast<const double2*>(Bc + o + W2);
+      const bool sw = (em.q[i] >> 11) & 1;
+      b00[i] = sw ? v0.y : v0.x;
+      b01[i] = sw ? v0.x : v0.y;
+      b10[i] = sw ? v1.y : v1.x;
+      b11[i] = sw ? v1.x : v1.y;
     }
   }
   const bool any = __any_sync(0xffffffffu, rot);
-  __syncwarp();
   if (!any) {
     PHASE_COUNT(8);  // profiling builds: rotation-free EVD steps
+#pragma unroll
+    for (int i = 0; i < QPL; ++i) {
+      if (em.q[i] & (1 << 13)) {
+        Bn[em.st[i][0] & 0xffff] = b00[i];
+        Bn[em.st[i][0] >> 16] = b01[i];
+        Bn[em.st[i][1] & 0xffff] = b10[i];
+        Bn[em.st[i][1] >> 16] = b11[i];
+      }
+    }
 #pragma unroll
     for (int k = 0; k < W2; ++k) y[rr_dest(k, W2)] = x[k];
     return false;
   }
+  __syncwarp();
 #pragma unroll
   for (int i = 0; i < QPL; ++i) {
-    if (qm.k[i] >= 0) {
-      const double2 gk = ws.cs[qm.k[i]], gl = ws.cs[qm.l[i]];
-      // columns (p_l, q_l): B G_l
-      const double c0 = fma(gl.y, b01[i], gl.x * b00[i]), c1 = fma(-gl.y, b00[i], gl.x * b01[i]);
-      const double d0 = fma(gl.y, b11[i], gl.x * b10[i]), d1 = fma(-gl.y, b10[i], gl.x * b11[i]);
-      // rows (p_k, q_k): G_k^T (B G_l)
-      const double e00 = fma(gk.y, d0, gk.x * c0), e01 = fma(gk.y, d1, gk.x * c1);
-      const double e10 = fma(-gk.y, c0, gk.x * d0), e11 = fma(-gk.y, c1, gk.x * d1);
-      const int pk = ak[i] & 0xffff, qk = ak[i] >> 16, pl = al[i] & 0xffff, ql = al[i] >> 16;
-      B[pk * BS + pl] = e00; B[pl * BS + pk] = e00;
-      B[pk * BS + ql] = e01; B[ql * BS + pk] = e01;
-      B[qk * BS + pl] = e10; B[pl * BS + qk] = e10;
-      B[qk * BS + ql] = e11; B[ql * BS + qk] = e11;
+    if (em.q[i] & (1 << 13)) {
+      const double2 gp = cs[(em.q[i] >> 16) & (NPR - 1)];
+      const bool own_lo = (em.q[i] >> 12) & 1;
+      const double rc = own_lo ? c : gp.x, rs = own_lo ? s : gp.y;  // rotation of the row pair
+      const double cc = own_lo ? gp.x : c, cs_ = own_lo ? gp.y : s;  // rotation of the column pair
+      // columns (2hi, 2hi+1): B G_hi
+      const double c0 = fma(cs_, b01[i], cc * b00[i]), c1 = fma(-cs_, b00[i], cc * b01[i]);
+      const double d0 = fma(cs_, b11[i], cc * b10[i]), d1 = fma(-cs_, b10[i], cc * b11[i]);
+      // rows (2lo, 2lo+1): G_lo^T (B G_hi)
+      Bn[em.st[i][0] & 0xffff] = fma(rs, d0, rc * c0);
+      Bn[em.st[i][0] >> 16] = fma(rs, d1, rc * c1);
+      Bn[em.st[i][1] & 0xffff] = fma(-rs, c0, rc * d0);
+      Bn[em.st[i][1] >> 16] = fma(-rs, c1, rc * d1);
     }
   }
   // J <- J G in slot order; outputs move to their next slots (register rename).
 #pragma unroll
   for (int k = 0; k < NPR; ++k) {
-    const double2 g = ws.cs[k];
+    const double2 g = cs[k];
     const double a = x[2 * k], b = x[2 * k + 1];
     y[rr_dest(2 * k, W2)] = fma(g.y, b, g.x * a);
     y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
   }
-  __syncwarp();
   return true;
 }
 
 // Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
 // rotated (A and V panels updated); counts inner sweeps into *inner.
 template <int W2>
-__device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, const int2* __restrict__ rrtab,
-                             double* Wm, int ld, int mrows,
+__device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, double* Wm, int ld, int mrows,
                              double* Vm, int ldv, int vrows, int I, int J, double tol2, int inner_cap,
                              int lane, int* inner) {
   using C = PairCfg<W2>;
   constexpr int CG = C::CG, BS = C::BS;
   PHASE_T0();
-  // (1) Gram B = P^T P, P = [W_I W_J] (Alg 1 l.5).
+  // (1) Gram B = P^T P, P = [W_I W_J] (Alg 1 l.5), upper triangle into the EVD layout.
+  double* B0 = ws.B;
+  double* B1 = ws.B + W2 * W2;
   {
     double acc[C::NTU][2];
     gram_tiles_async<W2>(ws, Wm, ld, mrows, I, J, lane, acc);
-    store_sym<W2>(ws.B, acc, lane, 0.0);
+    int t = 0;
+#pragma unroll
+    for (int a = 0; a < CG; ++a)
+#pragma unroll
+      for (int b = a; b < CG; ++b, ++t)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int row = 8 * a + (lane >> 2), col = 8 * b + 2 * (lane & 3) + e;
+          if (a != b || row <= col) B0[evd_phys<W2>(row, col)] = acc[t][e];
+        }
   }
   __syncwarp();
   PHASE_MARK(0);
   // (4) off-norm test on the Gram (Z6): skip the pair if every b_pq^2 <= tol^2 b_pp b_qq.
   bool need = false;
   {
-    const double bqq = (lane < W2) ? ws.B[lane * BS + lane] : 0.0;
+    const double bqq = (lane < W2) ? B0[evd_phys<W2>(lane, lane)] : 0.0;
 #pragma unroll 4
     for (int p = 0; p < W2 - 1; ++p) {
-      const double bpp = ws.B[p * BS + p];  // broadcast
-      const double bpq = (lane < W2) ? ws.B[p * BS + lane] : 0.0;
+      const double bpp = B0[evd_phys<W2>(p, p)];  // broadcast
+      const double bpq = (lane < W2 && lane > p) ? B0[evd_phys<W2>(p, lane)] : 0.0;
       const double ab = bpp * bqq;
       need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
     }
@@ -457,22 +498,29 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const QuadMap<W2>& qm, cons
   PHASE_MARK(1);
   PHASE_COUNT(7);
   if (!__any_sync(0xffffffffu, need)) return false;
-  // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, J accumulated in slot order.
+  // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, B and J in slot order.
+  EvdMap<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
+  em.init(lane);
   double ja[W2], jb[W2];
 #pragma unroll
   for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
   bool rotated = false;
   int isw = 0;
   for (; isw < inner_cap; ++isw) {
-    // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb, slots back in order.
-    constexpr int NPR = W2 / 2;
-    bool any = evd_step<W2>(ws, qm, rrtab, lane, tol2, ja, jb);
+    // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb / B1, slots back in order.
+    bool any = evd_step<W2>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+    __syncwarp();
     for (int r = 1; r < W2 - 1; r += 2) {
-      any |= evd_step<W2>(ws, qm, rrtab + r * NPR, lane, tol2, jb, ja);
-      any |= evd_step<W2>(ws, qm, rrtab + (r + 1) * NPR, lane, tol2, ja, jb);
+      any |= evd_step<W2>(B1, B0, ws.cs, em, lane, tol2, jb, ja);
+      __syncwarp();
+      any |= evd_step<W2>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+      __syncwarp();
     }
 #pragma unroll
     for (int s = 0; s < W2; ++s) ja[s] = jb[s];
+    double* tmp = B0;
+    B0 = B1;
+    B1 = tmp;
     rotated |= any;
     if (!any) break;
   }
@@ -563,11 +611,8 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __shared__ int s_inner[NW];
   __shared__ int s_grp[2 * NW];
   __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
-  __shared__ int2 s_rr[(W2 - 1) * (W2 / 2)];  // EVD round-robin table: (p, q) per step, pair
-  for (int e = tid; e < (W2 - 1) * (W2 / 2); e += NW * 32) {
-    const int r = e / (W2 / 2), k = e % (W2 / 2);
-    s_rr[e] = make_int2(rr_content(2 * k, r, W2), rr_content(2 * k + 1, r, W2));
-  }
+  __shared__ EvdMap<W2> s_em[32];     // inner-EVD work map per lane
+  if (tid < 32) s_em[tid].init(tid);
   if (tid < 4) s_flags[tid] = 0;
   if (tid < NW) s_inner[tid] = 0;
   if (tid < 2 * NW) s_grp[tid] = 0;
@@ -605,8 +650,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
   __syncthreads();
   const double tol2 = d.tol * d.tol;
-  QuadMap<W2> qm;
-  qm.init(lane);
+
 
   int sweep = 0;
   bool converged = false;
@@ -633,7 +677,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
           }
           __syncwarp();
           __threadfence_block();  // the previous owners' W / V writes are visible to every lane
-          rot_any |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
+          rot_any |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
           __syncwarp();           // every lane's W / V writes precede ...
           __threadfence_block();  // ... this fence, then the release (relaxed atomic store)
           if (lane == 0) {
@@ -676,7 +720,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
-                  mine |= process_pair<W2>(ws, qm, s_rr, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
+                  mine |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
                 }
                 named_bar(1 + grp, GS * 32);
               }
