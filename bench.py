@@ -305,7 +305,11 @@ def main():
         p = wc.plan(mm, nn)
         plans[(p["path"], p["variant"])] = p
     launches_per_step = len(plans) + 1
-    dominant = "l0_jacobi_kernel" if all(p["path"] == wc.PATH_L0 for p in plans.values()) else "l1_gram_kernel"
+    if all(p["path"] == wc.PATH_L0 for p in plans.values()):
+        dominant = "l0tp_kernel" if any(p["variant"] in wc.L0_TWO_PHASE_VARIANTS for p in plans.values()) \
+            else "l0_jacobi_kernel"
+    else:
+        dominant = "l1_gram_kernel"
 
     # roofline of the dominant kernel: algorithmic (textbook, sweep-normalised) flops per launch /
     # launch time. The step is one launch of it plus the tiny completion pass (ncu share in profiles/).

@@ -35,6 +35,16 @@ int l0_variant(int M, int N) {
   return 0;
 }
 
+// Two-phase Level-0 variant (l0_tp.cu), or 0: X and V_x time-share the registers of one CTA.
+int l0tp_variant(int M, int N) {
+#ifdef WCSVD_NO_TP
+  return 0;  // experiments: fused Level-0 kernel only
+#endif
+  if (N > 16 && N <= 32 && M > 48 && M <= kTP32MaxM) return kTP32;  // M <= 48: fused kL0_32s (latency)
+  if (N > 48 && N <= 64 && M <= kTP64MaxM) return kTP64;
+  return 0;
+}
+
 int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   std::memset(p, 0, sizeof(*p));
   p->m = m;
@@ -43,12 +53,13 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   p->M = std::max(m, n);
   p->N = std::min(m, n);
   p->cost = f_tb(p->M, p->N);
-  const int v = l0_variant(p->M, p->N);
+  const int tp = l0tp_variant(p->M, p->N);
+  const int v = tp ? tp : l0_variant(p->M, p->N);
   // Alg 2 l.2: "if SVD of A^k can be implemented entirely within SM" -> Level 0.
   if (v && (force_path == 0 || force_path == WCSVD_PATH_L0)) {
     p->path = WCSVD_PATH_L0;
     p->variant = v;
-    static const int np_of[] = {0, 8, 16, 32, 32, 48, 64};
+    static const int np_of[] = {0, 8, 16, 32, 32, 48, 64, 32, 64};
     p->n_pad = np_of[v];
     p->m_pad = p->M;
     return WCSVD_OK;
@@ -78,7 +89,7 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
 }
 
 size_t l1_bytes(const wcsvd_plan_t& p) {
-  if (p.path == WCSVD_PATH_L0) return 0;
+  if (p.path == WCSVD_PATH_L0) return (l0tp_park_bytes(p.variant, p.M) + 255) & ~size_t(255);
   const size_t b = sizeof(double) * ((size_t)p.m_pad * p.n_pad + (size_t)p.n_pad * p.n_pad);
   return (b + 255) & ~size_t(255);
 }
@@ -249,6 +260,8 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     if (p.path != WCSVD_PATH_L0) {
       d.W = reinterpret_cast<double*>(ws + l1_off[b]);
       d.Vw = d.W + (size_t)p.m_pad * p.n_pad;
+    } else if (l1_bytes(p)) {
+      d.W = reinterpret_cast<double*>(ws + l1_off[b]);  // two-phase L0 park buffer
     }
   }
   std::vector<int> h_order;
@@ -284,7 +297,9 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     const Bucket& bk = buckets[i];
     const int cnt = (int)bk.members.size();
     cudaStream_t st = (nbk > 1) ? side[i] : stream;
-    if (bk.path == WCSVD_PATH_L0)
+    if (bk.path == WCSVD_PATH_L0 && (bk.variant == kTP32 || bk.variant == kTP64))
+      e = launch_l0tp(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
+    else if (bk.path == WCSVD_PATH_L0)
       e = launch_l0(bk.variant, bk.withv, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
       e = launch_l1(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, st);

@@ -14,7 +14,11 @@ enum L0Variant {
   kL0_32s = 4,  // NP=32, G=2, R=1 (latency-bound small batches)
   kL0_48 = 5,   // NP=48, G=2, R=2
   kL0_64 = 6,   // NP=64, G=8, R=8
+  kTP32 = 7,    // two-phase (l0_tp.cu): NP=32 (layouts: l0_tp.cu TPCfg)
+  kTP64 = 8,    // two-phase (l0_tp.cu): NP=64
 };
+constexpr int kTP32MaxM = 128;  // planner limits of the two-phase variants (rows of the iterate)
+constexpr int kTP64MaxM = 64;
 
 // Level-1 Gram-path variants (pair panel width 2w, warps per CTA).
 enum L1Variant {
@@ -24,6 +28,10 @@ enum L1Variant {
 };
 
 cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
+
+cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
+                        cudaStream_t stream);
+size_t l0tp_park_bytes(int variant, int M);  // per-matrix park buffer (X and V_x registers), fp64
 
 cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, const int* order, int count,
                       int maxM, cudaStream_t stream);
