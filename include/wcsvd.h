@@ -98,6 +98,10 @@ typedef struct {
                               Gram path, Level 2 of the W-cycle path) */
   int wcycle_sweeps;       /* 0 = planner (2); cap on Level-2 sweeps per W-cycle super-pair */
   int inner_sweeps;        /* 0 = planner (1); cap on EVD sweeps per pair */
+  int pair_warps;          /* 0 = planner (1); 2 = two warps per column-block pair on the flat Gram
+                              path with w = 16 (ablation, SURVEY §8(f2) lanes-per-pair; results are
+                              as deterministic, but not bitwise equal to the 1-warp executor: the
+                              Gram partials are summed in another order) */
 } wcsvd_opts;
 
 WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,

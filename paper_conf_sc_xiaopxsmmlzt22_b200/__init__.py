@@ -47,7 +47,7 @@ class OptsT(ctypes.Structure):
                 ("info", ctypes.c_void_p), ("sweeps_inner", ctypes.c_void_p),
                 ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
                 ("force_path", ctypes.c_int), ("force_w", ctypes.c_int), ("wcycle_sweeps", ctypes.c_int),
-                ("inner_sweeps", ctypes.c_int)]
+                ("inner_sweeps", ctypes.c_int), ("pair_warps", ctypes.c_int)]
 
 
 _lib = None
@@ -118,7 +118,7 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
                     max_sweeps: int = 0, stream: int = 0, ldu=None, ldv=None, info_ptr: int = 0,
                     sweeps_inner_ptr: int = 0, workspace_ptr: int = 0, workspace_bytes: int = 0,
                     force_path: int = 0, force_w: int = 0, wcycle_sweeps: int = 0,
-                    inner_sweeps: int = 0, fp32: bool = False) -> None:
+                    inner_sweeps: int = 0, pair_warps: int = 0, fp32: bool = False) -> None:
     """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError.
     fp32=True calls wcsvd_batched_f32_ex (float data)."""
     m, n, lda = _arr_i32(m), _arr_i32(n), _arr_i32(lda)
@@ -138,6 +138,7 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
     opts.workspace = workspace_ptr or None
     opts.workspace_bytes = workspace_bytes
     opts.force_path, opts.force_w, opts.wcycle_sweeps, opts.inner_sweeps = force_path, force_w, wcycle_sweeps, inner_sweeps
+    opts.pair_warps = pair_warps
     fn = lib().wcsvd_batched_f32_ex if fp32 else lib().wcsvd_batched_ex
     rc = fn(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
             Sp.ctypes.data, Up.ctypes.data if Up is not None else None,

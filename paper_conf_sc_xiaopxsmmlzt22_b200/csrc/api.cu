@@ -171,6 +171,13 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     const int rc = plan_one(m[b], n[b], force_path, force_w, &plans[b]);
     if (rc != WCSVD_OK) return rc;
   }
+  // Ablation (wcsvd_opts.pair_warps = 2): the flat Gram path with 2w = 32 on the split executor
+  // (two warps per column-block pair, l1_gram.cu).
+  if (opts && opts->pair_warps == 2)
+    for (auto& p : plans)
+      if (p.path == WCSVD_PATH_GRAM && (p.variant == kL1_32x8 || p.variant == kL1_32x4))
+        p.variant = (p.variant == kL1_32x8) ? kL1S_32x16 : kL1S_32x8;
+  if (opts && opts->pair_warps != 0 && opts->pair_warps != 1 && opts->pair_warps != 2) return -12;
   // V_x (the square factor) is accumulated only if it is requested: as V when m >= n, as U when
   // m < n (§8(f4) values / U-only mode otherwise; the iteration itself is unchanged).
   std::vector<int> withv(batch);

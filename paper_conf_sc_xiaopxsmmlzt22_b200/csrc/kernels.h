@@ -25,6 +25,8 @@ enum L1Variant {
   kL1_16x4 = 11,  // 2w = 16, 4 warps
   kL1_32x4 = 12,  // 2w = 32, 4 warps
   kL1_32x8 = 13,  // 2w = 32, 8 warps
+  kL1S_32x8 = 14,   // 2w = 32, split executor (2 warps per pair): 4 pair groups, 8 warps
+  kL1S_32x16 = 15,  // 2w = 32, split executor: 8 pair groups, 16 warps
 };
 
 cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream);

@@ -148,10 +148,10 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 // Issue the copy of rows [r0, r0+16) of the 2w panel columns (offsets col_off[c] = pcol(c) * ld) into
 // ring stage `st`: W2 x 8 chunks of 16 B, W2/4 per lane.
 template <int W2>
-__device__ __forceinline__ void slab_issue(const WarpSmem<W2>& ws, const double* base, const int (&coff)[W2 / 4],
-                                           int r0, int st, int lane) {
+__device__ __forceinline__ void slab_issue(double* ring, const double* base, const int (&coff)[W2 / 4], int r0,
+                                           int st, int lane) {
   constexpr int SL = WarpSmem<W2>::SL;
-  double* dst = ws.ring + st * WarpSmem<W2>::SLAB;
+  double* dst = ring + st * WarpSmem<W2>::SLAB;
 #pragma unroll
   for (int i = 0; i < W2 / 4; ++i) {
     const int q = lane + 32 * i, c = q >> 3, h = q & 7;
@@ -166,12 +166,12 @@ __device__ __forceinline__ void slab_offsets(int (&coff)[W2 / 4], int I, int J, 
   for (int i = 0; i < W2 / 4; ++i) coff[i] = pcol<W2>((lane + 32 * i) >> 3, I, J) * ld;
 }
 
-// Upper tiles of P^T P for the global panel of pair (I, J): slabs stream through the ring while
-// the DMMAs consume the previous ones (no register staging, NSTAGE-1 slabs in flight).
-template <int W2>
-__device__ __forceinline__ void gram_tiles_async(const WarpSmem<W2>& ws, const double* base, int ld, int rows,
-                                                 int I, int J, int lane, double (&acc)[PairCfg<W2>::NTU][2]) {
-  constexpr int CG = W2 / 8, SL = WarpSmem<W2>::SL, NS = WarpSmem<W2>::NSTAGE;
+// Upper tiles of P^T P for the global panel of pair (I, J): slabs stream through the NS-stage ring
+// while the DMMAs consume the previous ones (no register staging, NS-1 slabs in flight).
+template <int W2, int NS>
+__device__ __forceinline__ void gram_tiles_async(double* ring, const double* base, int ld, int rows, int I, int J,
+                                                 int lane, double (&acc)[PairCfg<W2>::NTU][2]) {
+  constexpr int CG = W2 / 8, SL = WarpSmem<W2>::SL;
 #pragma unroll
   for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
   int coff[W2 / 4];
@@ -179,16 +179,16 @@ __device__ __forceinline__ void gram_tiles_async(const WarpSmem<W2>& ws, const d
   const int nslab = rows >> 4;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ws, base, coff, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2>(ring, base, coff, 16 * j, j, lane);
     cp_async_commit();
   }
   const int fo = (lane >> 2) * SL + (lane & 3);  // fragment offset inside a column group
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ws, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
-    const double* st = ws.ring + (sl % NS) * WarpSmem<W2>::SLAB;
+    const double* st = ring + (sl % NS) * WarpSmem<W2>::SLAB;
     double f[4][CG];
 #pragma unroll
     for (int u = 0; u < 4; ++u)
@@ -199,12 +199,12 @@ __device__ __forceinline__ void gram_tiles_async(const WarpSmem<W2>& ws, const d
   }
 }
 
-// X <- X * J' for the global panel of pair (I, J), slabs streamed through the ring; results are
-// stored straight to global memory (rows of a slab are read before they are overwritten).
-template <int W2>
-__device__ __forceinline__ void apply_rotation_async(const WarpSmem<W2>& ws, double* base, int ld, int rows,
-                                                     int I, int J, int lane, const double (&jf)[W2 / 4][W2 / 8]) {
-  constexpr int CG = W2 / 8, KK = W2 / 4, SL = WarpSmem<W2>::SL, NS = WarpSmem<W2>::NSTAGE;
+// X <- X * J' for the global panel of pair (I, J), slabs streamed through the NS-stage ring; results
+// are stored straight to global memory (rows of a slab are read before they are overwritten).
+template <int W2, int NS>
+__device__ __forceinline__ void apply_rotation_async(double* ring, double* base, int ld, int rows, int I, int J,
+                                                     int lane, const double (&jf)[W2 / 4][W2 / 8]) {
+  constexpr int CG = W2 / 8, KK = W2 / 4, SL = WarpSmem<W2>::SL;
   int coff[W2 / 4];
   slab_offsets<W2>(coff, I, J, ld, lane);
   int oc[CG][2];
@@ -215,16 +215,16 @@ __device__ __forceinline__ void apply_rotation_async(const WarpSmem<W2>& ws, dou
   const int nslab = rows >> 4;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ws, base, coff, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2>(ring, base, coff, 16 * j, j, lane);
     cp_async_commit();
   }
   const int fo = (lane & 3) * SL + (lane >> 2);  // A fragment: row l/4, column l%4
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ws, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
-    const double* st = ws.ring + (sl % NS) * WarpSmem<W2>::SLAB;
+    const double* st = ring + (sl % NS) * WarpSmem<W2>::SLAB;
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       double a[KK];
@@ -338,13 +338,14 @@ __device__ __forceinline__ int evd_phys_sym(int a, int b) {
   return (a <= b) ? evd_phys<W2>(a, b) : evd_phys<W2>(b, a);
 }
 
-// Lane-static EVD work map. Lane L works for pair k = L mod (w) (it evaluates that pair's rotation,
-// redundantly with the other lanes of the same k) and owns the off-diagonal quads {k, (k+d) mod w}
-// for its share of d = 1 .. w/2 (d = w/2 only from the lower k, so every unordered pair of pairs is
-// owned exactly once). Offsets are element offsets into a buffer.
-template <int W2>
+// Lane-static EVD work map. Lane L (of the NLANES lanes working on one EVD) works for pair
+// k = L mod (w) (it evaluates that pair's rotation, redundantly with the other lanes of the same k)
+// and owns the off-diagonal quads {k, (k+d) mod w} for its share of d = 1 .. w/2 (d = w/2 only from
+// the lower k, so every unordered pair of pairs is owned exactly once). Offsets are element offsets
+// into a buffer.
+template <int W2, int NLANES = 32>
 struct EvdMap {
-  static constexpr int NPR = W2 / 2, LPP = 32 / NPR, HALF = NPR / 2;
+  static constexpr int NPR = W2 / 2, LPP = NLANES / NPR, HALF = NPR / 2;
   static constexpr int QPL = (HALF + LPP - 1) / LPP;  // quads per lane
   int q[QPL];       // bits 0-10 load offset (row 2lo, aligned column pair), 11 swap, 12 own-is-lo,
                     // 13 valid, 16-19 partner pair
@@ -469,7 +470,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   double* B1 = ws.B + W2 * W2;
   {
     double acc[C::NTU][2];
-    gram_tiles_async<W2>(ws, Wm, ld, mrows, I, J, lane, acc);
+    gram_tiles_async<W2, WarpSmem<W2>::NSTAGE>(ws.ring, Wm, ld, mrows, I, J, lane, acc);
     int t = 0;
 #pragma unroll
     for (int a = 0; a < CG; ++a)
@@ -574,20 +575,389 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(3);
   // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J.
   __syncwarp();  // the ring aliases B: every lane holds its J' fragments before slabs land
-  apply_rotation_async<W2>(ws, Wm, ld, mrows, I, J, lane, jf);
+  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE>(ws.ring, Wm, ld, mrows, I, J, lane, jf);
   PHASE_MARK(4);
-  apply_rotation_async<W2>(ws, Vm, ldv, vrows, I, J, lane, jf);
+  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE>(ws.ring, Vm, ldv, vrows, I, J, lane, jf);
+  PHASE_MARK(5);
+  return true;
+}
+
+// ---- Split pair executor: two warps per column-block pair (2w = 32) ----
+// The EVD of one pair is issue- and latency-bound in a single warp (~600 instructions and a
+// sqrt/rsqrt chain per step, tools/evd_probe.cu), so a pair is owned by a group of two warps:
+// warp h of the group computes the Gram partial and the A / V update over its half of the rows,
+// holds the J columns of slot half h (slots 16h .. 16h+15, lane = row of J), and updates its half
+// of the off-diagonal quads of B (64-lane EvdMap). Both warps evaluate every rotation of a step
+// (bitwise the same numbers); warp 0 writes the diagonal blocks. One named barrier per EVD step
+// publishes B' and the two J values that cross between the column halves (the circle-method ring
+// moves slot 14 -> 16 and slot 17 -> 15, common.cuh). Twice the warps per SM at the same on-chip
+// footprint per matrix.
+constexpr int kSplitW2 = 32;
+constexpr int kSplitNS = 2;       // slab-ring stages per warp
+constexpr int kSplitSlab = 32 * 16;  // doubles per slab: 32 columns x 16 rows, XOR-swizzled rows (no pad)
+
+struct SplitSmem {
+  double* B;     // [2][W2 * W2] EVD ping-pong (slot layout); afterwards E = J^T J - I (stride BS)
+  double* S;     // [W2][BS] staged J
+  double* jf;    // [W2/4][W2/8][32] J' as DMMA B fragments (aliases S; written once S is consumed)
+  double* ring;  // this warp's [kSplitNS][kSplitSlab] slab ring (aliases B)
+  double* red;   // [NTU][2][32] Gram partials of warp 1 (inside warp 1's ring)
+  double2* cs;   // this warp's [W2 / 2] (c, s) of the current step
+  double* xch;   // [2 parity][2 halves][32] J values crossing between the column halves
+  // doubles: B [0, 2048), S [2048, 2048 + 32 * 33), jf [2048, 3072), rings [0, 2 * NS * slab)
+  __host__ __device__ static constexpr size_t region() {
+    constexpr size_t evd = (size_t)2 * kSplitW2 * kSplitW2 + (size_t)kSplitW2 * PairCfg<kSplitW2>::BS;
+    constexpr size_t rings = (size_t)2 * kSplitNS * kSplitSlab;
+    static_assert(rings <= 2 * kSplitW2 * kSplitW2, "rings must not reach the J' fragments");
+    return (evd > rings ? evd : rings) * sizeof(double);
+  }
+  __host__ __device__ static constexpr size_t bytes() {  // per group
+    return region() + 2 * sizeof(double2) * (kSplitW2 / 2) + sizeof(double) * 2 * 2 * 32;
+  }
+};
+
+// J columns of slot half HC: the value of global slot `gs` after the step goes to its next slot
+// (common.cuh rr_dest); within the half it is a register rename, across the halves it is sent.
+template <int HC>
+__device__ __forceinline__ void split_place(int gs, double v, double (&y)[16], double& send) {
+  const int dst = rr_dest(gs, kSplitW2) - 16 * HC;
+  if (dst >= 0 && dst < 16) y[dst] = v;
+  else send = v;
+}
+
+template <int HC>
+__device__ __forceinline__ bool evd_step_split(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
+                                               const EvdMap<kSplitW2, 64>& em, int lane, double tol2,
+                                               const double (&x)[16], double (&y)[16], double& send) {
+  constexpr int W2 = kSplitW2, NPR = W2 / 2, QPL = EvdMap<W2, 64>::QPL;
+  const double bpp = Bc[em.dld01 & 0xffff], bqq = Bc[em.dld01 >> 16], bpq = Bc[em.dld2];
+  double c, s, t;
+  const bool rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
+  if (lane < NPR) {
+    cs[lane] = make_double2(c, s);
+    if (HC == 0) {
+      Bn[em.dst01 & 0xffff] = rot ? fma(t, bpq, bpp) : bpp;
+      Bn[em.dst01 >> 16] = rot ? fma(-t, bpq, bqq) : bqq;
+      Bn[em.dst2] = rot ? 0.0 : bpq;
+    }
+  }
+  double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
+#pragma unroll
+  for (int i = 0; i < QPL; ++i) {
+    if (em.q[i] & (1 << 13)) {
+      const int o = em.q[i] & 0x7ff;
+      const double2 v0 = *reinterpret_cast<const double2*>(Bc + o);
+      const double2 v1 = *reinterpret_cast<const double2*>(Bc + o + W2);
+      const bool sw = (em.q[i] >> 11) & 1;
+      b00[i] = sw ? v0.y : v0.x;
+      b01[i] = sw ? v0.x : v0.y;
+      b10[i] = sw ? v1.y : v1.x;
+      b11[i] = sw ? v1.x : v1.y;
+    }
+  }
+  if (!__any_sync(0xffffffffu, rot)) {
+#pragma unroll
+    for (int i = 0; i < QPL; ++i) {
+      if (em.q[i] & (1 << 13)) {
+        Bn[em.st[i][0] & 0xffff] = b00[i];
+        Bn[em.st[i][0] >> 16] = b01[i];
+        Bn[em.st[i][1] & 0xffff] = b10[i];
+        Bn[em.st[i][1] >> 16] = b11[i];
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < 16; ++j) split_place<HC>(16 * HC + j, x[j], y, send);
+    return false;
+  }
+  __syncwarp();
+#pragma unroll
+  for (int i = 0; i < QPL; ++i) {
+    if (em.q[i] & (1 << 13)) {
+      const double2 gp = cs[(em.q[i] >> 16) & (NPR - 1)];
+      const bool own_lo = (em.q[i] >> 12) & 1;
+      const double rc = own_lo ? c : gp.x, rs = own_lo ? s : gp.y;
+      const double cc = own_lo ? gp.x : c, cs_ = own_lo ? gp.y : s;
+      const double c0 = fma(cs_, b01[i], cc * b00[i]), c1 = fma(-cs_, b00[i], cc * b01[i]);
+      const double d0 = fma(cs_, b11[i], cc * b10[i]), d1 = fma(-cs_, b10[i], cc * b11[i]);
+      Bn[em.st[i][0] & 0xffff] = fma(rs, d0, rc * c0);
+      Bn[em.st[i][0] >> 16] = fma(rs, d1, rc * c1);
+      Bn[em.st[i][1] & 0xffff] = fma(-rs, c0, rc * d0);
+      Bn[em.st[i][1] >> 16] = fma(-rs, c1, rc * d1);
+    }
+  }
+#pragma unroll
+  for (int kk = 0; kk < 8; ++kk) {
+    const double2 g = cs[8 * HC + kk];
+    const double a = x[2 * kk], b = x[2 * kk + 1];
+    split_place<HC>(16 * HC + 2 * kk, fma(g.y, b, g.x * a), y, send);
+    split_place<HC>(16 * HC + 2 * kk + 1, fma(-g.y, a, g.x * b), y, send);
+  }
+  return true;
+}
+
+// Split-executor panel streaming (2w = 32): the slab ring of gram_tiles_async / apply_rotation_async
+// with 16-double columns and the rows of column c stored XOR (4 (c mod 4)) (conflict-free fragment
+// reads without padding), panel addresses formed from the two block bases, and J' read from shared
+// memory (fragment order) instead of registers -- the executor runs at 128 registers per thread.
+__device__ __forceinline__ int slab_at(int c, int r) { return c * 16 + (r ^ (4 * (c & 3))); }
+
+struct SplitPanel {
+  const double* gI;  // this lane's copy source in block I: column I*16 + lane/8, rows 2 (lane%8) + {0,1}
+  const double* gJ;
+  size_t ld4;        // 4 columns
+  int so;            // this lane's slab offset of (column lane/8, rows 2 (lane%8)); + 64 i for column + 4 i
+  __device__ __forceinline__ SplitPanel(const double* base, int ld, int I, int J, int lane) {
+    gI = base + (size_t)(I * 16 + (lane >> 3)) * ld + 2 * (lane & 7);
+    gJ = base + (size_t)(J * 16 + (lane >> 3)) * ld + 2 * (lane & 7);
+    ld4 = (size_t)4 * ld;
+    so = slab_at(lane >> 3, 2 * (lane & 7));  // column lane/8 + 4 i has the same swizzle
+  }
+  __device__ __forceinline__ void issue(double* ring, int r0, int st) const {
+    double* dst = ring + st * kSplitSlab + so;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) cp_async16(dst + 64 * i, (i < 4 ? gI : gJ) + (i & 3) * ld4 + r0);
+  }
+};
+
+__device__ __forceinline__ void gram_split(double* ring, const double* base, int ld, int rows, int I, int J, int lane,
+                                           double (&acc)[PairCfg<kSplitW2>::NTU][2]) {
+  constexpr int W2 = kSplitW2, CG = W2 / 8, NS = kSplitNS;
+#pragma unroll
+  for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
+  const SplitPanel pn(base, ld, I, J, lane);
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) pn.issue(ring, 16 * j, j);
+    cp_async_commit();
+  }
+  // fragment (column 8 c + lane/4, row lane%4 + 4 u)
+  const int fc = (lane >> 2) * 16, fr = lane & 3, fx = (lane >> 2) & 3;
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) pn.issue(ring, 16 * (sl + NS - 1), (sl + NS - 1) % NS);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const double* st = ring + (sl % NS) * kSplitSlab + fc + fr;
+    double f[4][CG];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+      for (int c = 0; c < CG; ++c) f[u][c] = st[128 * c + 4 * (u ^ fx)];
+    gram_mma<W2>(acc, f);
+    __syncwarp();
+  }
+}
+
+__device__ __forceinline__ void apply_split(double* ring, double* base, int ld, int rows, int I, int J, int lane,
+                                            const double* __restrict__ jfs) {
+  constexpr int W2 = kSplitW2, CG = W2 / 8, KK = W2 / 4, NS = kSplitNS;
+  const SplitPanel pn(base, ld, I, J, lane);
+  // output element (row 16 sl + 8 h + lane/4, panel column 8 nb + 2 (lane%4) + e)
+  double* oI = base + (size_t)(I * 16 + 2 * (lane & 3)) * ld + (lane >> 2);
+  double* oJ = base + (size_t)(J * 16 + 2 * (lane & 3)) * ld + (lane >> 2);
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) pn.issue(ring, 16 * j, j);
+    cp_async_commit();
+  }
+  // A fragment (row 8 h + lane/4, column 4 kk + lane%4)
+  const int fa0 = slab_at(lane & 3, lane >> 2), fa1 = slab_at(lane & 3, 8 + (lane >> 2));
+  const double* jl = jfs + lane;
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) pn.issue(ring, 16 * (sl + NS - 1), (sl + NS - 1) % NS);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const double* st = ring + (sl % NS) * kSplitSlab;
+    double acc0[CG][2], acc1[CG][2];
+#pragma unroll
+    for (int nb = 0; nb < CG; ++nb) acc0[nb][0] = acc0[nb][1] = acc1[nb][0] = acc1[nb][1] = 0.0;
+#pragma unroll
+    for (int kk = 0; kk < KK; ++kk) {
+      const double a0 = st[64 * kk + fa0], a1 = st[64 * kk + fa1];
+#pragma unroll
+      for (int nb = 0; nb < CG; ++nb) {
+        const double bj = jl[(kk * CG + nb) * 32];
+        dmma884(acc0[nb], a0, bj);
+        dmma884(acc1[nb], a1, bj);
+      }
+    }
+#pragma unroll
+    for (int nb = 0; nb < CG; ++nb)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        double* o = (nb < 2 ? oI : oJ) + (size_t)(8 * (nb & 1) + e) * ld + 16 * sl;
+        __stcg(o, acc0[nb][e]);
+        __stcg(o + 8, acc1[nb][e]);
+      }
+    __syncwarp();
+  }
+}
+
+// Rows [0, h) go to warp 0 and [h, rows) to warp 1, h a multiple of 16.
+__device__ __forceinline__ int split_rows(int rows) { return 16 * (((rows >> 4) + 1) >> 1); }
+
+// One column-block pair (I, J) by the group's warp HC (bar_id: the group's named barrier).
+template <int HC>
+__device__ bool process_pair_split(const SplitSmem& ss, double* Wm, int ld, int mrows, double* Vm, int ldv,
+                                   int vrows, int I, int J, double tol2, int inner_cap, int lane, int bar_id,
+                                   int* inner) {
+  constexpr int W2 = kSplitW2;
+  using C = PairCfg<W2>;
+  constexpr int CG = C::CG, BS = C::BS, NTU = C::NTU;
+  double* B0 = ss.B;
+  double* B1 = ss.B + W2 * W2;
+  const int hm = split_rows(mrows);
+  const int r0 = HC ? hm : 0, nr = HC ? mrows - hm : hm;
+  PHASE_T0();
+  // (1) Gram B = P^T P (Alg 1 l.5): partials over each warp's rows, summed in a fixed order.
+  {
+    double acc[NTU][2];
+    gram_split(ss.ring, Wm + r0, ld, nr, I, J, lane, acc);
+    if (HC == 1) {
+#pragma unroll
+      for (int t = 0; t < NTU; ++t)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) ss.red[(2 * t + e) * 32 + lane] = acc[t][e];
+    }
+    named_bar(bar_id, 64);
+    if (HC == 0) {
+      int t = 0;
+#pragma unroll
+      for (int a = 0; a < CG; ++a)
+#pragma unroll
+        for (int b = a; b < CG; ++b, ++t)
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int row = 8 * a + (lane >> 2), col = 8 * b + 2 * (lane & 3) + e;
+            const double v = acc[t][e] + ss.red[(2 * t + e) * 32 + lane];
+            if (a != b || row <= col) B0[evd_phys<W2>(row, col)] = v;
+          }
+    }
+    named_bar(bar_id, 64);
+  }
+  PHASE_MARK(0);
+  // (4) off-norm test (Z6), evaluated identically by both warps.
+  bool need = false;
+  {
+    const double bqq = B0[evd_phys<W2>(lane, lane)];
+#pragma unroll 4
+    for (int p = 0; p < W2 - 1; ++p) {
+      const double bpp = B0[evd_phys<W2>(p, p)];
+      const double bpq = (lane > p) ? B0[evd_phys<W2>(p, lane)] : 0.0;
+      const double ab = bpp * bqq;
+      need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
+    }
+  }
+  PHASE_MARK(1);
+  PHASE_COUNT(7);
+  if (!__any_sync(0xffffffffu, need)) return false;
+  // (2) EVD of B (Alg 1 l.6), threshold parallel Jacobi split over the group.
+  EvdMap<W2, 64> em;
+  em.init(32 * HC + lane);
+  double ja[16], jb[16];
+#pragma unroll
+  for (int s = 0; s < 16; ++s) ja[s] = (lane == 16 * HC + s) ? 1.0 : 0.0;
+  constexpr int RECV = HC ? 0 : 15;  // local slot that receives the crossing value
+  double* xo = ss.xch + HC * 32 + lane;        // + parity * 64
+  const double* xi = ss.xch + (HC ^ 1) * 32 + lane;
+  int par = 0;
+  bool rotated = false;
+  int isw = 0;
+  for (; isw < inner_cap; ++isw) {
+    double send = 0.0;
+    bool any = evd_step_split<HC>(B0, B1, ss.cs, em, lane, tol2, ja, jb, send);
+    xo[par * 64] = send;
+    named_bar(bar_id, 64);
+    jb[RECV] = xi[par * 64];
+    par ^= 1;
+    for (int r = 1; r < W2 - 1; r += 2) {
+      any |= evd_step_split<HC>(B1, B0, ss.cs, em, lane, tol2, jb, ja, send);
+      xo[par * 64] = send;
+      named_bar(bar_id, 64);
+      ja[RECV] = xi[par * 64];
+      par ^= 1;
+      any |= evd_step_split<HC>(B0, B1, ss.cs, em, lane, tol2, ja, jb, send);
+      xo[par * 64] = send;
+      named_bar(bar_id, 64);
+      jb[RECV] = xi[par * 64];
+      par ^= 1;
+    }
+#pragma unroll
+    for (int s = 0; s < 16; ++s) ja[s] = jb[s];
+    double* tmp = B0;
+    B0 = B1;
+    B1 = tmp;
+    rotated |= any;
+    if (!any) break;
+  }
+  if (HC == 0) *inner += isw + (isw < inner_cap ? 1 : 0);
+  PHASE_MARK(2);
+  PHASE_COUNT(6);
+  if (!rotated) return false;
+  // Newton-Schulz (Z9(ii)): E = J^T J - I (warp 0), J' = J - J E / 2 (rows 16 HC .. 16 HC + 15).
+#pragma unroll
+  for (int s = 0; s < 16; ++s) ss.S[lane * BS + 16 * HC + s] = ja[s];
+  named_bar(bar_id, 64);
+  if (HC == 0) {
+    const double* ptr[CG];
+#pragma unroll
+    for (int c = 0; c < CG; ++c) ptr[c] = ss.S + (lane & 3) * BS + 8 * c + (lane >> 2);
+    double acc[NTU][2];
+    gram_tiles<W2>(ptr, W2, BS, acc);
+    store_sym<W2>(ss.B, acc, lane, 1.0);
+  }
+  named_bar(bar_id, 64);
+  {
+    double jn[2][CG][2];  // rows 8 (2 HC + ii) + lane/4 of J', columns 8 j + 2 (lane%4) + e
+#pragma unroll
+    for (int ii = 0; ii < 2; ++ii)
+#pragma unroll
+      for (int j = 0; j < CG; ++j) {
+        const int i = 2 * HC + ii;
+        double acc[2] = {0.0, 0.0};
+#pragma unroll
+        for (int kk = 0; kk < W2 / 4; ++kk)
+          dmma884(acc, ss.S[(8 * i + (lane >> 2)) * BS + 4 * kk + (lane & 3)],
+                  ss.B[(4 * kk + (lane & 3)) * BS + 8 * j + (lane >> 2)]);
+#pragma unroll
+        for (int e = 0; e < 2; ++e)
+          jn[ii][j][e] = fma(-0.5, acc[e], ss.S[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e]);
+      }
+    named_bar(bar_id, 64);  // S is consumed by both warps: the fragments may overwrite it
+    // J'[r][c] -> fragment (kk = r / 4, nb = c / 8) slot of lane 4 (c % 8) + r % 4
+#pragma unroll
+    for (int ii = 0; ii < 2; ++ii)
+#pragma unroll
+      for (int j = 0; j < CG; ++j)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int r = 8 * (2 * HC + ii) + (lane >> 2), c = 8 * j + 2 * (lane & 3) + e;
+          ss.jf[((r >> 2) * CG + j) * 32 + 4 * (c & 7) + (r & 3)] = jn[ii][j][e];
+        }
+  }
+  named_bar(bar_id, 64);
+  PHASE_MARK(3);
+  // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J over this warp's rows.
+  apply_split(ss.ring, Wm + r0, ld, nr, I, J, lane, ss.jf);
+  PHASE_MARK(4);
+  const int hv = split_rows(vrows);
+  apply_split(ss.ring, Vm + (HC ? hv : 0), ldv, HC ? vrows - hv : hv, I, J, lane, ss.jf);
   PHASE_MARK(5);
   return true;
 }
 
 }  // namespace
 
-template <int W2, int NW, typename TI>
-__global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
+template <int W2, int NW, typename TI, int GW>
+__global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
                                                              const int* __restrict__ order) {
   // TI: type of A, S, U, V in the caller's memory (double, or float for wcsvd_batched_f32); the
-  // iteration always runs on the fp64 working copy.
+  // iteration always runs on the fp64 working copy. GW: warps per column-block pair (1, or 2 =
+  // split executor, flat Gram path with 2w = 32 only).
+  static_assert(GW == 1 || (GW == 2 && W2 == kSplitW2 && NW % 2 == 0), "split executor: 2w = 32");
   using C = PairCfg<W2>;
   const MatDesc d = descs[order[blockIdx.x]];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -598,7 +968,17 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
 
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WarpSmem<W2> ws;
-  {
+  SplitSmem ss;
+  if constexpr (GW == 2) {
+    unsigned char* p = smem_raw + (warp >> 1) * SplitSmem::bytes();
+    ss.B = reinterpret_cast<double*>(p);
+    ss.S = ss.B + 2 * W2 * W2;
+    ss.jf = ss.S;
+    ss.ring = ss.B + (warp & 1) * kSplitNS * kSplitSlab;
+    ss.red = ss.B + kSplitNS * kSplitSlab;
+    ss.cs = reinterpret_cast<double2*>(p + SplitSmem::region()) + (warp & 1) * (W2 / 2);
+    ss.xch = reinterpret_cast<double*>(reinterpret_cast<double2*>(p + SplitSmem::region()) + W2);
+  } else {
     unsigned char* p = smem_raw + warp * WarpSmem<W2>::bytes();
     ws.B = reinterpret_cast<double*>(p);
     ws.S = ws.B + W2 * C::BS;
@@ -670,6 +1050,28 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     while (sweep < d.max_sweeps) {
       bool rot_any = false;
       for (int step = 0; step < nb - 1; ++step, ++gstep) {
+        if constexpr (GW == 2) {
+          // split executor: group g = warp / 2 owns pairs g, g + NW/2, ...; warp 0 of the group
+          // acquires / releases, the group's named barrier orders both warps around the pair.
+          const int grp = warp >> 1, hc = warp & 1, bar = 1 + grp;
+          for (int p = grp; p < nb / 2; p += NW / 2) {
+            const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
+            if (hc == 0 && lane == 0) {
+              while (atomicAdd(&blk_ver[I], 0) < gstep || atomicAdd(&blk_ver[J], 0) < gstep) __nanosleep(20);
+            }
+            named_bar(bar, 64);
+            __threadfence_block();
+            rot_any |= hc ? process_pair_split<1>(ss, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, bar, &my_inner)
+                          : process_pair_split<0>(ss, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, bar, &my_inner);
+            __syncwarp();
+            __threadfence_block();
+            named_bar(bar, 64);
+            if (hc == 0 && lane == 0) {
+              atomicExch(&blk_ver[I], gstep + 1);
+              atomicExch(&blk_ver[J], gstep + 1);
+            }
+          }
+        } else {
         for (int p = warp; p < nb / 2; p += NW) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
           if (lane == 0) {  // acquire: relaxed atomic reads, then a fence
@@ -685,6 +1087,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
             atomicExch(&blk_ver[J], gstep + 1);
           }
         }
+        }
       }
       ++sweep;
       if (rot_any && lane == 0) s_flags[sweep & 1] = 1;
@@ -694,7 +1097,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
       if (tid == 0) s_flags[sweep & 1] = 0;
       if (!any) { converged = true; break; }
     }
-  } else if (!nonfinite) {
+  } else if (GW == 1 && !nonfinite) {
     // W-cycle (Alg 2 l.12-14; Step 3; Fig 3-4): Level-1 super-blocks
     // of width w1 = d.w are paired round-robin; each super-pair panel [A_I A_J] (M x 2 w1) fits no
     // on-chip EVD, so it recurses to Level 2: block Jacobi with w2 = d.w2 (the EVD width W2/2) over
@@ -828,12 +1231,12 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
 }
 
-template <int W2, int NW, typename TI>
+template <int W2, int NW, typename TI, int GW>
 static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
-  size_t smem = NW * WarpSmem<W2>::bytes();
+  size_t smem = (GW == 2) ? (NW / 2) * SplitSmem::bytes() : NW * WarpSmem<W2>::bytes();
   const size_t fin = 3 * 8 * 1024;  // finalisation arrays alias the warp buffers
   if (smem < fin) smem = fin;
-  auto kern = l1_gram_kernel<W2, NW, TI>;
+  auto kern = l1_gram_kernel<W2, NW, TI, GW>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<count, NW * 32, smem, stream>>>(descs, order);
@@ -843,9 +1246,11 @@ static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count
 template <typename TI>
 static cudaError_t launch_l1_v(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
   switch (variant) {
-    case kL1_16x4: return launch_l1_t<16, 4, TI>(descs, order, count, stream);
-    case kL1_32x4: return launch_l1_t<32, 4, TI>(descs, order, count, stream);
-    case kL1_32x8: return launch_l1_t<32, 8, TI>(descs, order, count, stream);
+    case kL1_16x4: return launch_l1_t<16, 4, TI, 1>(descs, order, count, stream);
+    case kL1_32x4: return launch_l1_t<32, 4, TI, 1>(descs, order, count, stream);
+    case kL1_32x8: return launch_l1_t<32, 8, TI, 1>(descs, order, count, stream);
+    case kL1S_32x8: return launch_l1_t<32, 8, TI, 2>(descs, order, count, stream);
+    case kL1S_32x16: return launch_l1_t<32, 16, TI, 2>(descs, order, count, stream);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -5,7 +5,7 @@ sys.path.insert(0, '.')
 import workloads
 import paper_conf_sc_xiaopxsmmlzt22_b200 as wc
 name = sys.argv[1] if len(sys.argv) > 1 else "C2"
-batch = int(sys.argv[2]) if len(sys.argv) > 2 else None
+batch = int(sys.argv[2]) if len(sys.argv) > 2 and sys.argv[2] else None
 kw = json.loads(sys.argv[3]) if len(sys.argv) > 3 else {}
 cfg = workloads.get_config(name, batch)
 t0 = time.time()
