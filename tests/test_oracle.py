@@ -248,3 +248,23 @@ def test_c1_workload_spectrum_matches_prescription():
     for k in range(5):
         r = oracle.svd(cfg.make(k))
         assert np.abs(r.S - cfg.spectrum(k)).max() <= 20 * U53
+
+
+def test_oracle_table7_standins(capsys):
+    # the Table VII stand-ins (sizes and condition numbers of the paper's picks,
+    # PAPER.md:469-476; kappa 3.1 .. 8.08e15) -- pinned to their prescribed spectra (known by
+    # construction, exact up to the fp64 rounding of A) and to the invariants; the sweep counts are
+    # printed as the reference column of the GPU robustness table (tools/robustness.py).
+    cfg = workloads.table7_config()
+    mats = cfg.matrices()
+    S, U, V, info = oracle.svd_batch(mats)
+    for k, A in enumerate(mats):
+        s_true = cfg.spectrum(k)
+        assert info[k] > 0
+        assert np.abs(S[k] - s_true).max() <= 1e-13
+        # north_star's bars (the residual is formed in fp64 from fp64-rounded factors)
+        assert compare.residual(A, S[k], U[k], V[k]) <= 1e-12
+        assert compare.orthogonality(U[k]) <= 1e-11 and compare.orthogonality(V[k]) <= 1e-11
+    with capsys.disabled():
+        print("\noracle sweeps on the Table VII stand-ins:",
+              {workloads.TABLE7[k][0]: int(info[k]) for k in range(len(mats))})

@@ -1,0 +1,70 @@
+"""SURVEY §8(f3) measurement: the Table VII / Fig 15 analogue on B200.
+
+For the five synthetic stand-ins (workloads.table7_config: the sizes and condition numbers of the
+paper's SuiteSparse picks), report the outer sweeps the CUDA path needs (planner path, forced EVD
+widths w = 8 / 16, forced W-cycle) next to the CPU oracle's (row-cyclic, long double) and the paper's
+own counts (context: different matrices, different GPU and stopping rule), plus the final errors
+against the prescribed spectrum (the CPU oracle's sweep counts on the same inputs come from
+tests/test_oracle.py::test_oracle_table7_standins, which prints them; tools/ never runs the oracle). For
+impcol_d (the Fig 15 matrix) it also records the error after each sweep (max_sweeps = s returns the
+iterate after s sweeps): max |sigma - sigma_true| / sigma_1 and ||U^T U - I||_max, the Fig 15(a)
+analogue. Prints one JSON object.
+"""
+import json
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import workloads  # noqa: E402
+import paper_conf_sc_xiaopxsmmlzt22_b200 as wc  # noqa: E402
+
+KNOBS = {"planner": {}, "w=8": {"force_path": wc.PATH_GRAM, "force_w": 8},
+         "w=16": {"force_path": wc.PATH_GRAM, "force_w": 16},
+         "wcycle(w1=64,w2=16)": {"force_path": wc.PATH_WCYCLE, "force_w": 16}}
+
+
+def errors(A, S, U, V, s_true):
+    return {"sigma_err": float(np.abs(S - s_true).max() / s_true[0]),
+            "residual": float(np.linalg.norm(A - (U * S) @ V.T) / np.linalg.norm(A)),
+            "orth_U": float(np.abs(U.T @ U - np.eye(U.shape[1])).max()),
+            "orth_V": float(np.abs(V.T @ V - np.eye(V.shape[1])).max())}
+
+
+def main():
+    cfg = workloads.table7_config()
+    mats = cfg.matrices()
+    dev = torch.device("cuda:0")
+    As = [torch.from_numpy(a).to(dev) for a in mats]
+    out = {"gpu": torch.cuda.get_device_name(0), "matrices": []}
+    runs = {}
+    for knob, kw in KNOBS.items():
+        S, U, V, info = wc.svd_batched(As, return_info=True, **kw)
+        torch.cuda.synchronize()
+        runs[knob] = ([s.cpu().numpy() for s in S], [u.cpu().numpy() for u in U], [v.cpu().numpy() for v in V],
+                      info.cpu().numpy())
+    for k, (name, m, n, kappa, p_cusolver, p_wcycle) in enumerate(workloads.TABLE7):
+        rec = {"name": name, "size": f"{m}x{n}", "kappa": kappa,
+               "paper_sweeps": {"cuSOLVER": p_cusolver, "W-cycle SVD": p_wcycle}}
+        for knob, (S, U, V, info) in runs.items():
+            rec[knob] = {"sweeps": int(info[k]), **errors(mats[k], S[k], U[k], V[k], cfg.spectrum(k))}
+        out["matrices"].append(rec)
+        print(name, {kn: rec[kn]["sweeps"] for kn in KNOBS}, file=sys.stderr)
+    # Fig 15(a) analogue: error after each sweep, impcol_d (k = 1), planner path and W-cycle
+    curve = {}
+    for knob in ("planner", "wcycle(w1=64,w2=16)"):
+        pts = []
+        for s in range(1, runs[knob][3][1] + 1):
+            S, U, V, info = wc.svd_batched([As[1]], return_info=True, max_sweeps=s, **KNOBS[knob])
+            torch.cuda.synchronize()
+            e = errors(mats[1], S[0].cpu().numpy(), U[0].cpu().numpy(), V[0].cpu().numpy(), cfg.spectrum(1))
+            pts.append({"sweeps": s, "sigma_err": e["sigma_err"], "orth_U": e["orth_U"]})
+        curve[knob] = pts
+    out["impcol_d_error_per_sweep"] = curve
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()
