@@ -262,25 +262,24 @@ def main():
     ms_step = ms / args.steps
     value = world * B * args.steps / (ms * 1e-3)
 
-    # ---- e2e: host (pinned) inputs -> H2D -> library call -> D2H of S, U, V; inside the timing ----
+    # ---- e2e: the public end-to-end call with HOST buffers (wcsvd_batched_host): pinned inputs ->
+    # H2D -> kernels -> D2H of S, U, V, pipelined over chunks inside the library; inside the timing ----
     if uniform:
-        S_h = torch.empty(out[0].shape, dtype=torch.float64).pin_memory()
-        U_h = torch.empty(out[1].shape, dtype=torch.float64).pin_memory()
-        V_h = torch.empty(out[2].shape, dtype=torch.float64).pin_memory()
-        A_dev = torch.empty_like(A)
+        k_ = min(sizes[0])
+        S_h = torch.empty(B, k_, dtype=torch.float64).pin_memory()
+        U_h = torch.empty(B, k_, sizes[0][0], dtype=torch.float64).pin_memory()
+        V_h = torch.empty(B, k_, sizes[0][1], dtype=torch.float64).pin_memory()
 
         def e2e_step():
-            A_dev.copy_(A_h, non_blocking=True)
-            call(A_dev)
-            S_h.copy_(out[0], non_blocking=True)
-            U_h.copy_(out[1], non_blocking=True)
-            V_h.copy_(out[2], non_blocking=True)
+            wc.svd_batched_host(A_h, out=(S_h, U_h, V_h))
     else:
+        ks_ = [min(mm, nn) for (mm, nn) in sizes]
+        out_h = ([torch.empty(k, dtype=torch.float64).pin_memory() for k in ks_],
+                 [torch.empty(k, mm, dtype=torch.float64).pin_memory() for k, (mm, _) in zip(ks_, sizes)],
+                 [torch.empty(k, nn, dtype=torch.float64).pin_memory() for k, (_, nn) in zip(ks_, sizes)])
+
         def e2e_step():
-            Ad = [a.to(dev, non_blocking=True) for a in A_h]
-            S, U, V, _ = call(Ad)
-            for t in S + U + V:
-                t.to("cpu", non_blocking=True)
+            wc.svd_batched_host(A_h, out=out_h)
     e2e_step()
     barrier()
     ee0 = torch.cuda.Event(enable_timing=True)

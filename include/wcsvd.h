@@ -121,6 +121,26 @@ WCSVD_API int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const 
                                    const int* lda, float* const* S, float* const* U, float* const* V,
                                    float tol, int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
 
+/* wcsvd_batched_host -- the same factorisation with HOST buffers (the end-to-end call: host -> device
+ * copies, the iteration and device -> host copies all inside).
+ *   A[b], S[b], U[b], V[b]: HOST pointers (column-major, lda / ldu / ldv as in wcsvd_batched). Page-locked
+ *     memory gives full copy/compute overlap; pageable memory is accepted (the copies then block the
+ *     calling thread per chunk and overlap less).
+ *   U, V: NULL, or an array of non-NULL pointers for every matrix (-7 if some entries are NULL).
+ *   opts: as wcsvd_batched_ex, except that opts->info is a HOST int[batch]; workspace is ignored.
+ * Pipeline: a uniform batch is cut into up to 6 contiguous chunks; chunk c is copied in (stream 1),
+ * factored on one of two compute streams, and copied out (stream 2) while chunk c+1 is being copied in /
+ * factored, through two device staging sets (stream-ordered allocation). A mixed-size batch is one chunk
+ * (its size buckets overlap each other instead). Host blocks of consecutive matrices that are adjacent
+ * and packed (ld = rows) move as one copy (per matrix if the runtime refuses a merged range).
+ * Ordered after prior work on `stream`; SYNCHRONOUS: returns when every output is in host memory.
+ * Results are bitwise those of wcsvd_batched on the same inputs (per-matrix determinism).
+ * Errors: the argument checks of wcsvd_batched (returned before anything is enqueued); ENOMEM if the
+ * staging cannot be allocated; ECUDA on a failed copy or launch. */
+WCSVD_API int wcsvd_batched_host(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                                 double* const* S, double* const* U, double* const* V, double tol,
+                                 int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
+
 /* Bytes of device workspace wcsvd_batched_ex needs for this batch (host-only, no CUDA call). */
 WCSVD_API size_t wcsvd_workspace_size(int batch, const int* m, const int* n);
 

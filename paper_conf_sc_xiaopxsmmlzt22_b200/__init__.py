@@ -17,7 +17,7 @@ from typing import Sequence
 
 import numpy as np
 
-__all__ = ["svd_batched", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
+__all__ = ["svd_batched", "svd_batched_host", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
            "PATH_L0", "PATH_GRAM", "PATH_WCYCLE", "L0_TWO_PHASE_VARIANTS", "library_path"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -73,6 +73,8 @@ def lib() -> ctypes.CDLL:
     L.wcsvd_batched_ex.restype = I
     L.wcsvd_batched_f32_ex.argtypes = [I, P, P, P, P, P, P, P, ctypes.c_float, I, P, ctypes.POINTER(OptsT)]
     L.wcsvd_batched_f32_ex.restype = I
+    L.wcsvd_batched_host.argtypes = [I, P, P, P, P, P, P, P, D, I, P, ctypes.POINTER(OptsT)]
+    L.wcsvd_batched_host.restype = I
     L.wcsvd_workspace_size.argtypes = [I, P, P]
     L.wcsvd_workspace_size.restype = ctypes.c_size_t
     L.wcsvd_status_string.argtypes = [I]
@@ -222,6 +224,93 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
                     [u.data_ptr() for u in Ub] if Ub is not None else None,
                     tol=tol, max_sweeps=max_sweeps, stream=stream,
                     info_ptr=info.data_ptr() if info is not None else 0, fp32=(dt == torch.float32), **kw)
+    Us = [u.T for u in Ub] if Ub is not None else None
+    Vs = [v.T for v in Vb] if Vb is not None else None
+    return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)
+
+
+def _host_call(ms, ns, a_ptrs, s_ptrs, u_ptrs, v_ptrs, tol, max_sweeps, info, kw):
+    opts = OptsT()
+    opts.struct_size = ctypes.sizeof(OptsT)
+    opts.info = info.ctypes.data if info is not None else None
+    for key in ("force_path", "force_w", "wcycle_sweeps", "inner_sweeps", "pair_warps"):
+        setattr(opts, key, int(kw.pop(key, 0)))
+    if kw:
+        raise TypeError(f"unexpected arguments {sorted(kw)}")
+    import torch
+    stream = torch.cuda.current_stream().cuda_stream
+    mm, nn = _arr_i32(ms), _arr_i32(ns)
+    a_ptr, s_ptr = _arr_ptr(a_ptrs), _arr_ptr(s_ptrs)
+    u_ptr = _arr_ptr(u_ptrs) if u_ptrs is not None else None
+    v_ptr = _arr_ptr(v_ptrs) if v_ptrs is not None else None
+    rc = lib().wcsvd_batched_host(len(mm), mm.ctypes.data, nn.ctypes.data, a_ptr.ctypes.data, mm.ctypes.data,
+                                  s_ptr.ctypes.data, u_ptr.ctypes.data if u_ptr is not None else None,
+                                  v_ptr.ctypes.data if v_ptr is not None else None, float(tol), int(max_sweeps),
+                                  stream or None, ctypes.byref(opts))
+    _check(rc)
+
+
+def svd_batched_host(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = True,
+                     return_info: bool = False, out=None, **kw):
+    """End-to-end batched SVD of HOST fp64 data (wcsvd_batched_host): the host -> device copies, the
+    iteration and the device -> host copies run inside one library call, pipelined over chunks (the
+    copies overlap the kernels). A: host tensor [B, m, n] or a list of host 2-D tensors (sizes may
+    differ); pin them (``pin_memory()``) for full overlap. Returns host (S, U, V) shaped like
+    ``svd_batched``'s (U, V are transposed views of row-major [k, m] / [k, n] buffers), pinned when A
+    is. ``out`` = (S, Ubuf, Vbuf) preallocated host buffers: tensors [B, k], [B, k, m], [B, k, n] (tensor
+    form) or lists of [k], [k, m], [k, n] (list form). Synchronous. With return_info, also the per-matrix info as a numpy int32 array.
+    """
+    import torch
+
+    if not torch.cuda.is_available():
+        raise WcsvdError(WCSVD_ECUDA, "no CUDA device (this library has no CPU fallback)")
+    info = None
+    if isinstance(A, torch.Tensor):
+        if A.dim() != 3 or A.dtype != torch.float64 or A.is_cuda:
+            raise ValueError("A must be a float64 host tensor [B, m, n]")
+        A = A.contiguous()
+        B, m, n = A.shape
+        k = min(m, n)
+        if out is not None:
+            S, Ubuf, Vbuf = out
+        else:
+            pin = A.is_pinned()
+            S = torch.empty(B, k, dtype=A.dtype, pin_memory=pin)
+            Ubuf = torch.empty(B, k, m, dtype=A.dtype, pin_memory=pin) if compute_uv else None
+            Vbuf = torch.empty(B, k, n, dtype=A.dtype, pin_memory=pin) if compute_uv else None
+        info = np.zeros(B, dtype=np.int32) if return_info else None
+        idx = np.arange(B, dtype=np.uint64)
+        es = np.uint64(8)
+        # column-major view (as svd_batched): the library factors A^T (n x m, lda = n); its U is our V
+        _host_call(np.full(B, n), np.full(B, m), A.data_ptr() + idx * (es * np.uint64(m * n)),
+                   S.data_ptr() + idx * (es * np.uint64(k)),
+                   (Vbuf.data_ptr() + idx * (es * np.uint64(k * n))) if Vbuf is not None else None,
+                   (Ubuf.data_ptr() + idx * (es * np.uint64(k * m))) if Ubuf is not None else None,
+                   tol, max_sweeps, info, kw)
+        U = Ubuf.transpose(1, 2) if Ubuf is not None else None
+        V = Vbuf.transpose(1, 2) if Vbuf is not None else None
+        return (S, U, V, info) if return_info else (S, U, V)
+    As = [a.contiguous() for a in A]
+    for a in As:
+        if a.dim() != 2 or a.dtype != torch.float64 or a.is_cuda:
+            raise ValueError("each matrix must be a 2-D float64 host tensor")
+    B = len(As)
+    if B == 0:
+        return ([], [], []) if not return_info else ([], [], [], None)
+    pin = all(a.is_pinned() for a in As)
+    ms = [a.shape[0] for a in As]
+    ns = [a.shape[1] for a in As]
+    ks = [min(x, y) for x, y in zip(ms, ns)]
+    if out is not None:  # lists (S, Ubuf, Vbuf) of host buffers [k], [k, m], [k, n]
+        Ss, Ub, Vb = out
+    else:
+        Ss = [torch.empty(k, dtype=torch.float64, pin_memory=pin) for k in ks]
+        Ub = [torch.empty(k, mm, dtype=torch.float64, pin_memory=pin) for k, mm in zip(ks, ms)] if compute_uv else None
+        Vb = [torch.empty(k, nn, dtype=torch.float64, pin_memory=pin) for k, nn in zip(ks, ns)] if compute_uv else None
+    info = np.zeros(B, dtype=np.int32) if return_info else None
+    _host_call(ns, ms, [a.data_ptr() for a in As], [s.data_ptr() for s in Ss],
+               [v.data_ptr() for v in Vb] if Vb is not None else None,
+               [u.data_ptr() for u in Ub] if Ub is not None else None, tol, max_sweeps, info, kw)
     Us = [u.T for u in Ub] if Ub is not None else None
     Vs = [v.T for v in Vb] if Vb is not None else None
     return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)

@@ -82,3 +82,22 @@ def test_plan_is_pure_and_transposes_wide():
     assert wc.plan(40, 24) == p1
     for (m, n) in [(32, 32), (64, 64)]:
         assert wc.plan(m, n)["path"] == wc.PATH_L0
+
+
+def test_host_entry_point_validates_before_any_cuda_call():
+    # wcsvd_batched_host (end-to-end call with host buffers): LAPACK-style argument codes, returned
+    # before anything is allocated or enqueued (so they work without a GPU).
+    import ctypes
+    L = wc.lib()
+    P = ctypes.c_void_p
+    one = np.array([1], dtype=np.int32)
+    bad = np.array([0], dtype=np.int32)
+    buf = np.zeros(4)
+    ptr = np.array([buf.ctypes.data], dtype=np.uint64)
+    assert L.wcsvd_batched_host(-1, None, None, None, None, None, None, None, 0.0, 0, None, None) == -1
+    assert L.wcsvd_batched_host(0, None, None, None, None, None, None, None, 0.0, 0, None, None) == 0
+    assert L.wcsvd_batched_host(1, bad.ctypes.data, one.ctypes.data, ptr.ctypes.data, one.ctypes.data,
+                                ptr.ctypes.data, None, None, 0.0, 0, None, None) == -2
+    big = np.array([2048], dtype=np.int32)
+    assert L.wcsvd_batched_host(1, big.ctypes.data, one.ctypes.data, ptr.ctypes.data, big.ctypes.data,
+                                ptr.ctypes.data, None, None, 0.0, 0, None, None) == -100
