@@ -427,12 +427,21 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // device staging offsets (packed per matrix, in batch order)
   std::vector<size_t> oA(batch), oS(batch), oU(batch), oV(batch);
   std::vector<int> kk(batch), ldu_v(batch), ldv_v(batch);
-  // chunks: contiguous index ranges of ~equal textbook cost (6 when the batch allows). A mixed-size
+  // chunks: contiguous index ranges of ~equal textbook cost. A mixed-size
   // batch is one chunk: its cost-sorted buckets run concurrently only within one call (chunked, the
   // largest matrices of every chunk would each bound a chunk's duration: C5 e2e 776 vs 891 /s).
   bool uniform = true;
   for (int b = 1; b < batch && uniform; ++b) uniform = (m[b] == m[0] && n[b] == n[0]);
-  const int nch = uniform ? std::max(1, std::min(batch, 6)) : 1;
+  // chunk count measured on B200 (C2: 1/6/8/12 chunks -> 36.4/28.9/28.6/25.3 ms; C4: 516/421/413/457 ms):
+  // ~1.5 resident waves per chunk -- 12 for Level-0 shapes (4 CTAs/SM), 8 for the Gram path
+  int nch = 1;
+  if (uniform) {
+    wcsvd_plan_t p0;
+    const int want = (plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
+                      p0.path == WCSVD_PATH_L0) ? 12 : 8;
+    nch = std::max(1, std::min(batch, want));
+  }
+  if (const char* env = std::getenv("WCSVD_HOST_CHUNKS")) nch = std::max(1, std::min(batch, std::atoi(env)));  // experiments
   double tot = 0;
   for (int b = 0; b < batch; ++b) tot += f_tb(std::max(m[b], n[b]), std::min(m[b], n[b]));
   std::vector<int> cb{0};
