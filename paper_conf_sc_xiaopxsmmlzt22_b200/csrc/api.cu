@@ -347,15 +347,28 @@ struct HostRun {
   int b0, nb;       // the matrices of the run (per-matrix fallback)
 };
 
-// Group matrices [b0, b1) into copy runs: consecutive packed matrices whose host blocks are adjacent.
+// True if the whole batch of this array is one packed block in host memory (a [B, ...] array): only
+// then are adjacent matrices merged into one copy (separately allocated page-locked buffers that happen
+// to be adjacent may not be spanned by one copy).
+template <typename Ptr>
+bool whole_adjacent(int batch, Ptr host, const int* rows, const int* cols, const int* ld) {
+  for (int b = 1; b < batch; ++b)
+    if (ld[b - 1] != rows[b - 1] ||
+        reinterpret_cast<const double*>(host[b - 1]) + (size_t)rows[b - 1] * cols[b - 1] != reinterpret_cast<const double*>(host[b]))
+      return false;
+  return ld[0] == rows[0];
+}
+
+// Group matrices [b0, b1) into copy runs: consecutive packed matrices whose host blocks are adjacent
+// (when `merge`), else one run per matrix.
 template <typename Ptr>
 std::vector<HostRun> host_runs(int b0, int b1, const std::vector<size_t>& off, Ptr host, const int* rows,
-                               const int* cols, const int* ld) {
+                               const int* cols, const int* ld, bool merge) {
   std::vector<HostRun> runs;
   for (int b = b0; b < b1; ++b) {
     const size_t el = (size_t)rows[b] * cols[b];
     const bool packed = ld[b] == rows[b];
-    if (!runs.empty() && packed && runs.back().elems &&
+    if (merge && !runs.empty() && packed && runs.back().elems &&
         reinterpret_cast<const double*>(runs.back().src) + runs.back().elems == reinterpret_cast<const double*>(host[b]) &&
         runs.back().dst_off + runs.back().elems == off[b]) {
       runs.back().elems += el;
@@ -469,6 +482,11 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     mxA = std::max(mxA, a); mxS = std::max(mxS, s); mxU = std::max(mxU, u); mxV = std::max(mxV, v);
     mxB = std::max(mxB, cb[c + 1] - cb[c]);
   }
+  const std::vector<int> ones(batch, 1);  // S[b] is a k x 1 block
+  const bool mergeA = whole_adjacent(batch, A, m, n, lda);
+  const bool mergeS = whole_adjacent(batch, S, kk.data(), ones.data(), kk.data());
+  const bool mergeU = wantU && whole_adjacent(batch, U, m, kk.data(), ldu_v.data());
+  const bool mergeV = wantV && whole_adjacent(batch, V, n, kk.data(), ldv_v.data());
   const size_t setE = mxA + mxS + mxU + mxV;  // doubles per staging set
   const size_t setB = (setE * sizeof(double) + sizeof(int) * (size_t)mxB + 255) & ~size_t(255);
   double* dbuf = nullptr;
@@ -510,19 +528,18 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     stage(c, dA, dS, dU, dV, dI);
     cudaError_t x = cudaStreamWaitEvent(s_out, ev_cp[st], 0);
     {
-      std::vector<int> ones(batch, 1);  // S[b] is a k x 1 block
-      for (const HostRun& r : host_runs(b0, b1, oS, S, kk.data(), ones.data(), kk.data())) {
+      for (const HostRun& r : host_runs(b0, b1, oS, S, kk.data(), ones.data(), kk.data(), mergeS)) {
         if (x != cudaSuccess) break;
         x = copy_run(r, false, dS, oS, S, kk.data(), ones.data(), kk.data(), s_out);
       }
     }
     if (wantU)
-      for (const HostRun& r : host_runs(b0, b1, oU, U, m, kk.data(), ldu_v.data())) {
+      for (const HostRun& r : host_runs(b0, b1, oU, U, m, kk.data(), ldu_v.data(), mergeU)) {
         if (x != cudaSuccess) break;
         x = copy_run(r, false, dU, oU, U, m, kk.data(), ldu_v.data(), s_out);
       }
     if (wantV)
-      for (const HostRun& r : host_runs(b0, b1, oV, V, n, kk.data(), ldv_v.data())) {
+      for (const HostRun& r : host_runs(b0, b1, oV, V, n, kk.data(), ldv_v.data(), mergeV)) {
         if (x != cudaSuccess) break;
         x = copy_run(r, false, dV, oV, V, n, kk.data(), ldv_v.data(), s_out);
       }
@@ -538,7 +555,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     stage(c, dA, dS, dU, dV, dI);
     // H2D into staging set st, once the D2H of chunk c-2 (same set) has drained it
     if (c >= 2) e = cudaStreamWaitEvent(s_in, ev_out[st], 0);
-    for (const HostRun& r : host_runs(b0, b1, oA, A, m, n, lda)) {
+    for (const HostRun& r : host_runs(b0, b1, oA, A, m, n, lda, mergeA)) {
       if (e != cudaSuccess) break;
       e = copy_run(r, true, dA, oA, A, m, n, lda, s_in);
     }

@@ -51,8 +51,12 @@ __device__ unsigned long long g_phase_cycles[12];
 #define PHASE_COUNT(i) (void)0
 #endif
 
+// Named barrier over `count` threads (whole warps). The non-.aligned form (barrier.sync, not bar.sync):
+// the two warps of a split pair group reach it from different code (process_pair_split<0> / <1>), which
+// the .aligned form does not allow; the warp is reconverged first (lane-0-only spins precede some uses).
 __device__ __forceinline__ void named_bar(int id, int count) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+  __syncwarp();
+  asm volatile("barrier.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
 
 template <int W2>

@@ -1,4 +1,5 @@
-"""Small mixed batch for compute-sanitizer runs (L0 variants, L1 flat w=8/16, W-cycle)."""
+"""Small mixed batch for compute-sanitizer runs (L0 variants, L1 flat w=8/16, W-cycle, the split pair
+executor, the host-buffer pipeline)."""
 import sys
 import numpy as np, torch
 sys.path.insert(0, '.')
@@ -11,6 +12,16 @@ kw = {}
 if mode == "wcycle":
     mats = [mats[4], mats[6]]
     kw = dict(force_path=wc.PATH_WCYCLE)
+if mode == "split":  # two warps per column-block pair (w = 16 shapes)
+    mats = [mats[4], mats[6], workloads.gaussian(workloads.matrix_rng(778, 0), 300, 256)]
+    kw = dict(pair_warps=2)
+if mode == "host":  # wcsvd_batched_host: chunked copy / compute pipeline, uniform and mixed
+    A = torch.from_numpy(np.stack([workloads.gaussian(workloads.matrix_rng(779, i), 64, 64) for i in range(40)]))
+    S, U, V, info = wc.svd_batched_host(A.pin_memory(), return_info=True)
+    print("info", info[:8])
+    S, U, V, info = wc.svd_batched_host([torch.from_numpy(a).pin_memory() for a in mats], return_info=True)
+    print("info", info)
+    sys.exit(0)
 S, U, V, info = wc.svd_batched([torch.from_numpy(a).cuda() for a in mats], return_info=True, **kw)
 torch.cuda.synchronize()
 print("info", info.cpu().numpy())
