@@ -50,3 +50,43 @@ def test_host_values_only_and_preallocated_out():
     assert torch.equal(S0, S1)
     Sd, Ud, Vd, _ = _dev(A)
     assert torch.equal(S1, Sd) and torch.equal(U1, Ud) and torch.equal(V1, Vd)
+
+
+def test_host_strided_ld_and_host_info_through_the_c_abi():
+    # column-major host blocks with lda > m and ldu / ldv > m / n (the 2-D copy path), pageable numpy
+    # memory, per-matrix host info; compared bitwise with the device entry point.
+    import ctypes
+    rng = workloads.matrix_rng(880, 0)
+    shapes = [(70, 50), (50, 70), (130, 120), (64, 64)]
+    L = wc.lib()
+    B = len(shapes)
+    m = np.array([s[0] for s in shapes], dtype=np.int32)
+    n = np.array([s[1] for s in shapes], dtype=np.int32)
+    k = np.minimum(m, n)
+    lda, ldu, ldv = m + 3, m + 5, n + 2
+    A = [np.asfortranarray(np.vstack([rng.standard_normal((mm, nn)), np.zeros((3, nn))])) for mm, nn in shapes]
+    S = [np.zeros(kk) for kk in k]
+    U = [np.zeros((lu, kk), order="F") for lu, kk in zip(ldu, k)]
+    V = [np.zeros((lv, kk), order="F") for lv, kk in zip(ldv, k)]
+    ptrs = lambda xs: np.array([x.ctypes.data for x in xs], dtype=np.uint64)
+    pa, ps, pu, pv = ptrs(A), ptrs(S), ptrs(U), ptrs(V)
+    info = np.zeros(B, dtype=np.int32)
+    opts = wc.OptsT()
+    opts.struct_size = ctypes.sizeof(wc.OptsT)
+    opts.ldu, opts.ldv, opts.info = ldu.ctypes.data, ldv.ctypes.data, info.ctypes.data
+    rc = L.wcsvd_batched_host(B, m.ctypes.data, n.ctypes.data, pa.ctypes.data, lda.ctypes.data, ps.ctypes.data,
+                              pu.ctypes.data, pv.ctypes.data, 0.0, 0, None, ctypes.byref(opts))
+    assert rc == 0 and (info > 0).all()
+    for b, (mm, nn) in enumerate(shapes):
+        # the device entry point on the same column-major matrix (row-major [n, m] = column-major m x n)
+        kk = int(k[b])
+        Ad = torch.from_numpy(np.ascontiguousarray(A[b][:mm, :].T)).cuda()
+        Sd = torch.empty(kk, dtype=torch.float64, device="cuda")
+        Ud = torch.empty(kk, mm, dtype=torch.float64, device="cuda")
+        Vd = torch.empty(kk, nn, dtype=torch.float64, device="cuda")
+        wc.svd_batched_raw([mm], [nn], [Ad.data_ptr()], [mm], [Sd.data_ptr()], [Ud.data_ptr()], [Vd.data_ptr()],
+                           stream=torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        assert np.array_equal(S[b], Sd.cpu().numpy())
+        assert np.array_equal(U[b][:mm, :], Ud.cpu().numpy().T) and np.array_equal(V[b][:nn, :], Vd.cpu().numpy().T)
+        assert not U[b][mm:, :].any() and not V[b][nn:, :].any()  # rows past m / n untouched
