@@ -16,8 +16,7 @@ SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitize
 
 @pytest.mark.parametrize("tool,mode", [("memcheck", "mixed"), ("racecheck", "mixed"), ("racecheck", "wcycle"),
                                        ("synccheck", "mixed"), ("initcheck", "mixed"), ("racecheck", "split"),
-                                       ("memcheck", "split"), ("synccheck", "split"), ("synccheck", "wcycle"),
-                                       ("memcheck", "host")])
+                                       ("synccheck", "split"), ("synccheck", "wcycle"), ("memcheck", "host")])
 def test_sanitizer_clean(tool, mode):
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not available")

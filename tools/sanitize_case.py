@@ -13,7 +13,7 @@ if mode == "wcycle":
     mats = [mats[4], mats[6]]
     kw = dict(force_path=wc.PATH_WCYCLE)
 if mode == "split":  # two warps per column-block pair (w = 16 shapes)
-    mats = [mats[4], mats[6], workloads.gaussian(workloads.matrix_rng(778, 0), 300, 256)]
+    mats = [mats[4], workloads.gaussian(workloads.matrix_rng(778, 0), 120, 160)]
     kw = dict(pair_warps=2)
 if mode == "host":  # wcsvd_batched_host: chunked copy / compute pipeline, uniform and mixed
     A = torch.from_numpy(np.stack([workloads.gaussian(workloads.matrix_rng(779, i), 64, 64) for i in range(40)]))
