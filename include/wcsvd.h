@@ -128,7 +128,7 @@ WCSVD_API int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const 
  *     calling thread per chunk and overlap less).
  *   U, V: NULL, or an array of non-NULL pointers for every matrix (-7 if some entries are NULL).
  *   opts: as wcsvd_batched_ex, except that opts->info is a HOST int[batch]; workspace is ignored.
- * Pipeline: a uniform batch is cut into up to 12 (Level 0) or 8 (Gram path) contiguous chunks; chunk c
+ * Pipeline: a uniform batch is cut into contiguous chunks (~500 matrices for Level 0, 8 for the Gram path); chunk c
  * is copied in (stream 1), factored on one of two compute streams, and copied out (stream 2) while chunk
  * c+1 is being copied in / factored, through two device staging sets (stream-ordered allocation). A mixed-size batch is one chunk
  * (its size buckets overlap each other instead). Host blocks of consecutive matrices that are adjacent

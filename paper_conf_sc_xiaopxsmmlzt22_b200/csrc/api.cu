@@ -445,13 +445,16 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // largest matrices of every chunk would each bound a chunk's duration: C5 e2e 776 vs 891 /s).
   bool uniform = true;
   for (int b = 1; b < batch && uniform; ++b) uniform = (m[b] == m[0] && n[b] == n[0]);
-  // chunk count measured on B200 (C2: 1/6/8/12 chunks -> 36.4/28.9/28.6/25.3 ms; C4: 516/421/413/457 ms):
-  // ~1.5 resident waves per chunk -- 12 for Level-0 shapes (4 CTAs/SM), 8 for the Gram path
+  // chunk count measured on B200: Level 0 (C2, 10,000 x 64^2) 1/6/12/16/20/24/32 chunks -> 36.4/28.9/
+  // 25.6/28.8/23.2/25.2/29.8 ms, i.e. best near 500 matrices per chunk (just under one resident wave of
+  // 4 CTAs x 148 SMs, two chunks in flight); Gram path (C3 / C4) 8 chunks (C3 4/6/8/12 -> 262/263/250/
+  // 268 ms, C4 1/6/8/12 -> 516/421/413/457 ms)
   int nch = 1;
   if (uniform) {
     wcsvd_plan_t p0;
-    const int want = (plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
-                      p0.path == WCSVD_PATH_L0) ? 12 : 8;
+    const bool l0 = plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
+                    p0.path == WCSVD_PATH_L0;
+    const int want = l0 ? std::min(32, (batch + 499) / 500) : 8;
     nch = std::max(1, std::min(batch, want));
   }
   if (const char* env = std::getenv("WCSVD_HOST_CHUNKS")) nch = std::max(1, std::min(batch, std::atoi(env)));  // experiments

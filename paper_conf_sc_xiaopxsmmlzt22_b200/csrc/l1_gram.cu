@@ -27,6 +27,10 @@
 #include "rotation.cuh"
 #include "wcsvd.h"
 
+#ifndef WCSVD_L1_NSTAGE
+#define WCSVD_L1_NSTAGE 3
+#endif
+
 namespace wcsvd {
 
 namespace {
@@ -78,7 +82,7 @@ struct WarpSmem {
   int2* pq;     // [NPR]    (p, q) original indices of the step's pairs
   double* ring;  // [NSTAGE][W2][SL] cp.async slab ring for the Gram / update panels (aliases B, S)
   static constexpr int SL = 20;      // ring column stride (doubles): 16 rows + 4 pad (conflict-free fragments)
-  static constexpr int NSTAGE = 3;   // slabs in flight
+  static constexpr int NSTAGE = WCSVD_L1_NSTAGE;  // slabs in flight (ring stages)
   static constexpr int SLAB = W2 * SL;  // doubles per slab
   __host__ __device__ static constexpr size_t region() {
     return (2 * W2 * PairCfg<W2>::BS > NSTAGE * SLAB ? 2 * W2 * PairCfg<W2>::BS : NSTAGE * SLAB) * sizeof(double);

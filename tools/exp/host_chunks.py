@@ -19,6 +19,6 @@ def t(f, r=3):
 print(name, "H2D A ms", round(t(lambda: A_d.copy_(A_h, non_blocking=True)), 2),
       "D2H U+V ms", round(t(lambda: (U_h.copy_(U_d, non_blocking=True), V_h.copy_(V_d, non_blocking=True))), 2))
 print("device call ms", round(t(lambda: wc.svd_batched(A_d)), 2))
-for c in [1, 2, 3, 4, 6, 8, 12]:
+for c in [int(x) for x in (sys.argv[2].split(',') if len(sys.argv) > 2 else '1,2,3,4,6,8,12'.split(','))]:
     os.environ["WCSVD_HOST_CHUNKS"] = str(c)
     print("chunks", c, "e2e ms", round(t(lambda: wc.svd_batched_host(A_h, out=(S_h, U_h, V_h))), 2), flush=True)
