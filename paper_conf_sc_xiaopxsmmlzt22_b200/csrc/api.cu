@@ -19,6 +19,8 @@ namespace wcsvd {
 namespace {
 
 constexpr int kMaxDim = 1024;
+constexpr int kHostSets = 4;         // max device staging sets of the host-buffer pipeline
+constexpr int kHostSetsDefault = 3;
 
 double f_tb(int M, int N) { return 0.5 * N * (N - 1.0) * (8.0 * M + 6.0 * N); }
 
@@ -448,13 +450,15 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // chunk count measured on B200: Level 0 (C2, 10,000 x 64^2) 1/6/12/16/20/24/32 chunks -> 36.4/28.9/
   // 25.6/28.8/23.2/25.2/29.8 ms, i.e. best near 500 matrices per chunk (just under one resident wave of
   // 4 CTAs x 148 SMs, two chunks in flight); Gram path (C3 / C4) 8 chunks (C3 4/6/8/12 -> 262/263/250/
-  // 268 ms, C4 1/6/8/12 -> 516/421/413/457 ms)
+  // 268 ms, C4 1/6/8/12 -> 516/421/413/457 ms) with two staging sets; with three (r01g, e2e matrices/s):
+  // C2 20 chunks 424k (2 sets) / 465k (3) / 443k (4), 32 chunks 420k; C3 8 / 16 chunks 8455 / 8467;
+  // C4 8 / 16 chunks 9804 / 10634 -> Gram path 16 chunks
   int nch = 1;
   if (uniform) {
     wcsvd_plan_t p0;
     const bool l0 = plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
                     p0.path == WCSVD_PATH_L0;
-    const int want = l0 ? std::min(32, (batch + 499) / 500) : 8;
+    const int want = l0 ? std::min(32, (batch + 499) / 500) : 16;
     nch = std::max(1, std::min(batch, want));
   }
   if (const char* env = std::getenv("WCSVD_HOST_CHUNKS")) nch = std::max(1, std::min(batch, std::atoi(env)));  // experiments
@@ -492,20 +496,24 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   const bool mergeV = wantV && whole_adjacent(batch, V, n, kk.data(), ldv_v.data());
   const size_t setE = mxA + mxS + mxU + mxV;  // doubles per staging set
   const size_t setB = (setE * sizeof(double) + sizeof(int) * (size_t)mxB + 255) & ~size_t(255);
+  // staging sets: chunk c uses set c % NSET, so its H2D waits only for the D2H of chunk c - NSET (with two
+  // sets, D2H(c-2) + H2D(c) had to fit inside one chunk's kernel time: bubbles at ~500-matrix chunks)
+  int NSET = kHostSetsDefault;
+  if (const char* env = std::getenv("WCSVD_HOST_SETS")) NSET = std::max(2, std::min(kHostSets, std::atoi(env)));  // experiments
+  NSET = std::min(NSET, std::max(2, C));
   double* dbuf = nullptr;
-  if (cudaMallocAsync(reinterpret_cast<void**>(&dbuf), 2 * setB, stream) != cudaSuccess) {
+  if (cudaMallocAsync(reinterpret_cast<void**>(&dbuf), NSET * setB, stream) != cudaSuccess) {
     cudaGetLastError();
     return WCSVD_ENOMEM;
   }
   int* h_info = opts ? opts->info : nullptr;  // HOST int[batch] for this entry point
   cudaStream_t s_in = nullptr, s_out = nullptr, s_cp[2] = {nullptr, nullptr};
-  cudaEvent_t ev_start = nullptr, ev_in[2] = {nullptr, nullptr}, ev_cp[2] = {nullptr, nullptr},
-              ev_out[2] = {nullptr, nullptr};
+  cudaEvent_t ev_start = nullptr, ev_in[kHostSets] = {}, ev_cp[kHostSets] = {}, ev_out[kHostSets] = {};
   cudaError_t e = cudaStreamCreateWithFlags(&s_in, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&s_out, cudaStreamNonBlocking);
-  for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
-    e = cudaStreamCreateWithFlags(&s_cp[i], cudaStreamNonBlocking);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_in[i], cudaEventDisableTiming);
+  for (int i = 0; i < 2 && e == cudaSuccess; ++i) e = cudaStreamCreateWithFlags(&s_cp[i], cudaStreamNonBlocking);
+  for (int i = 0; i < NSET && e == cudaSuccess; ++i) {
+    e = cudaEventCreateWithFlags(&ev_in[i], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_cp[i], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_out[i], cudaEventDisableTiming);
   }
@@ -517,7 +525,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   int rc = WCSVD_OK;
   const size_t es = sizeof(double);
   auto stage = [&](int c, double*& dA, double*& dS, double*& dU, double*& dV, int*& dI) {
-    unsigned char* base = reinterpret_cast<unsigned char*>(dbuf) + (c & 1) * setB;
+    unsigned char* base = reinterpret_cast<unsigned char*>(dbuf) + (c % NSET) * setB;
     dA = reinterpret_cast<double*>(base);
     dS = dA + mxA;
     dU = dS + mxS;
@@ -525,7 +533,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     dI = reinterpret_cast<int*>(dV + mxV);
   };
   auto d2h = [&](int c) -> cudaError_t {
-    const int b0 = cb[c], b1 = cb[c + 1], st = c & 1;
+    const int b0 = cb[c], b1 = cb[c + 1], st = c % NSET;
     double *dA, *dS, *dU, *dV;
     int* dI;
     stage(c, dA, dS, dU, dV, dI);
@@ -552,19 +560,19 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     return x;
   };
   for (int c = 0; c < C && e == cudaSuccess && rc == WCSVD_OK; ++c) {
-    const int b0 = cb[c], b1 = cb[c + 1], cnt = b1 - b0, st = c & 1;
+    const int b0 = cb[c], b1 = cb[c + 1], cnt = b1 - b0, st = c % NSET, cs = c & 1;
     double *dA, *dS, *dU, *dV;
     int* dI;
     stage(c, dA, dS, dU, dV, dI);
-    // H2D into staging set st, once the D2H of chunk c-2 (same set) has drained it
-    if (c >= 2) e = cudaStreamWaitEvent(s_in, ev_out[st], 0);
+    // H2D into staging set st, once the D2H of chunk c-NSET (same set) has drained it
+    if (c >= NSET) e = cudaStreamWaitEvent(s_in, ev_out[st], 0);
     for (const HostRun& r : host_runs(b0, b1, oA, A, m, n, lda, mergeA)) {
       if (e != cudaSuccess) break;
       e = copy_run(r, true, dA, oA, A, m, n, lda, s_in);
     }
     if (e == cudaSuccess) e = cudaEventRecord(ev_in[st], s_in);
-    // kernels on compute stream st
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(s_cp[st], ev_in[st], 0);
+    // kernels on compute stream cs
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(s_cp[cs], ev_in[st], 0);
     if (e != cudaSuccess) break;
     std::vector<const double*> pA(cnt);
     std::vector<double*> pS(cnt), pU(wantU ? cnt : 0), pV(wantV ? cnt : 0);
@@ -590,9 +598,9 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     }
     rc = batched_impl<double>(cnt, m + b0, n + b0, pA.data(), ld_.data(), pS.data(), wantU ? pU.data() : nullptr,
                               wantV ? pV.data() : nullptr, tol, max_sweeps,
-                              reinterpret_cast<wcsvd_stream_t>(s_cp[st]), &o);
+                              reinterpret_cast<wcsvd_stream_t>(s_cp[cs]), &o);
     if (rc != WCSVD_OK) break;
-    e = cudaEventRecord(ev_cp[st], s_cp[st]);
+    e = cudaEventRecord(ev_cp[st], s_cp[cs]);
     // D2H of the previous chunk now (a copy to pageable host memory returns only when it is done, so
     // it is issued after this chunk's kernels are queued), this chunk's after the loop / next round
     if (e == cudaSuccess && c >= 1) e = d2h(c - 1);
@@ -624,12 +632,13 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   }
   cudaFreeAsync(dbuf, stream);
   const cudaError_t es2 = cudaStreamSynchronize(stream);
-  for (int i = 0; i < 2; ++i) {
+  for (int i = 0; i < NSET; ++i) {
     if (ev_in[i]) cudaEventDestroy(ev_in[i]);
     if (ev_cp[i]) cudaEventDestroy(ev_cp[i]);
     if (ev_out[i]) cudaEventDestroy(ev_out[i]);
-    if (s_cp[i]) cudaStreamDestroy(s_cp[i]);
   }
+  for (int i = 0; i < 2; ++i)
+    if (s_cp[i]) cudaStreamDestroy(s_cp[i]);
   if (ev_start) cudaEventDestroy(ev_start);
   if (s_in) cudaStreamDestroy(s_in);
   if (s_out) cudaStreamDestroy(s_out);

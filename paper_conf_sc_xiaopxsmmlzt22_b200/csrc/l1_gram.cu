@@ -15,7 +15,7 @@
 // "slot" order so that every rotation writes fixed registers (common.cuh). Threshold rotations make
 // J = I exactly once B is diagonal to tol; the EVD is capped at inner_cap sweeps
 // (Z8); J is re-orthogonalised by one Newton-Schulz step J <- J - J (J^T J - I)/2 before it is
-// applied (Z9(ii)). A pair whose Gram is already diagonal to tol is skipped with no writes; a
+// applied (Z9(ii); R-NS: a build option keeps it off). A pair whose Gram is already diagonal to tol is skipped with no writes; a
 // sweep in which every pair is skipped ends the iteration (Z6, Z9(iii)).
 #include <cuda_runtime.h>
 
@@ -27,6 +27,13 @@
 #include "rotation.cuh"
 #include "wcsvd.h"
 
+// Newton-Schulz cleanup of J before it is applied. -DWCSVD_L1_NS=0 drops it (ablation,
+// DESIGN.md §3 R-NS): 4-5% faster on Level 1 (B200, r01g: C3 229 -> 220 ms, C4 364 -> 345 ms, C5 2.93 ->
+// 2.82 s) but sigma / residual errors ~50x larger on the Table VII stand-ins (up to 5.5e-13 / 9.3e-13 on
+// the W-cycle, against the 1e-12 bar), so the default keeps it.
+#ifndef WCSVD_L1_NS
+#define WCSVD_L1_NS 1
+#endif
 #ifndef WCSVD_L1_NSTAGE
 #define WCSVD_L1_NSTAGE 3
 #endif
@@ -537,12 +544,13 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(2);
   PHASE_COUNT(6);
   if (!rotated) return false;
-  // Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2.
+  // Stage J; Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2.
   if (lane < W2) {
 #pragma unroll
     for (int s = 0; s < W2; ++s) ws.S[lane * BS + s] = ja[s];
   }
   __syncwarp();
+#if WCSVD_L1_NS
   {
     const double* ptr[CG];
 #pragma unroll
@@ -575,11 +583,15 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
 #pragma unroll
       for (int e = 0; e < 2; ++e) ws.B[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e] = jn[i][j][e];
   __syncwarp();
+  const double* jsrc = ws.B;
+#else
+  const double* jsrc = ws.S;  // ablation build (-DWCSVD_L1_NS=0): J applied without the cleanup step
+#endif
   double jf[W2 / 4][CG];
 #pragma unroll
   for (int kk = 0; kk < W2 / 4; ++kk)
 #pragma unroll
-    for (int nb = 0; nb < CG; ++nb) jf[kk][nb] = ws.B[(4 * kk + (lane & 3)) * BS + 8 * nb + (lane >> 2)];
+    for (int nb = 0; nb < CG; ++nb) jf[kk][nb] = jsrc[(4 * kk + (lane & 3)) * BS + 8 * nb + (lane >> 2)];
   PHASE_MARK(3);
   // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J.
   __syncwarp();  // the ring aliases B: every lane holds its J' fragments before slabs land
