@@ -442,9 +442,9 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // device staging offsets (packed per matrix, in batch order)
   std::vector<size_t> oA(batch), oS(batch), oU(batch), oV(batch);
   std::vector<int> kk(batch), ldu_v(batch), ldv_v(batch);
-  // chunks: contiguous index ranges of ~equal textbook cost. A mixed-size
-  // batch is one chunk: its cost-sorted buckets run concurrently only within one call (chunked, the
-  // largest matrices of every chunk would each bound a chunk's duration: C5 e2e 776 vs 891 /s).
+  // chunks: contiguous index ranges of ~equal textbook cost. A mixed-size batch takes few chunks: its
+  // cost-sorted buckets run concurrently only within one call, and the largest matrices of every chunk
+  // bound that chunk's duration (two staging sets: C5 e2e 776 with 8 chunks vs 891 with one).
   bool uniform = true;
   for (int b = 1; b < batch && uniform; ++b) uniform = (m[b] == m[0] && n[b] == n[0]);
   // chunk count measured on B200: Level 0 (C2, 10,000 x 64^2) 1/6/12/16/20/24/32 chunks -> 36.4/28.9/
@@ -453,7 +453,9 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // 268 ms, C4 1/6/8/12 -> 516/421/413/457 ms) with two staging sets; with three (r01g, e2e matrices/s):
   // C2 20 chunks 424k (2 sets) / 465k (3) / 443k (4), 32 chunks 420k; C3 8 / 16 chunks 8455 / 8467;
   // C4 8 / 16 chunks 9804 / 10634 -> Gram path 16 chunks
-  int nch = 1;
+  // mixed batches: 3 equal-cost chunks when large (C5, three staging sets, r01i: 1/2/3/4/6 chunks -> e2e
+  // 892/906/927/745/620 matrices/s; beyond 3 every chunk is bounded by its own largest matrices)
+  int nch = batch >= 300 ? 3 : 1;
   if (uniform) {
     wcsvd_plan_t p0;
     const bool l0 = plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
