@@ -41,6 +41,20 @@ def test_host_mixed_list_bitwise_equals_device():
     assert np.array_equal(info, infod.cpu().numpy())
 
 
+def test_host_mixed_chunked_bitwise_equals_device():
+    # >= 300 mixed-size matrices take the chunked path (3 equal-cost chunks, three staging sets)
+    rng = np.random.default_rng(77)
+    shapes = [(int(rng.integers(8, 97)), int(rng.integers(8, 97))) for _ in range(320)]
+    mats = [torch.from_numpy(workloads.gaussian(workloads.matrix_rng(900, k), m, n)).pin_memory()
+            for k, (m, n) in enumerate(shapes)]
+    S, U, V, info = wc.svd_batched_host(mats, return_info=True)
+    Sd, Ud, Vd, infod = wc.svd_batched([a.cuda() for a in mats], return_info=True)
+    torch.cuda.synchronize()
+    for k in range(len(mats)):
+        assert torch.equal(S[k], Sd[k].cpu()) and torch.equal(U[k], Ud[k].cpu()) and torch.equal(V[k], Vd[k].cpu()), k
+    assert np.array_equal(info, infod.cpu().numpy()) and (info > 0).all()
+
+
 def test_host_values_only_and_preallocated_out():
     mats = workloads.get_config("C3", batch=20).matrices()
     A = torch.from_numpy(np.stack(mats)).pin_memory()
