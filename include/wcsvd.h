@@ -15,8 +15,11 @@
  *  - fp64, column-major, economy SVD: S[k] descending, U m x k, V n x k.
  *  - Ownership: the caller owns A, S, U, V (DEVICE memory) and every host array; host arrays are
  *    consumed before the call returns and may be freed immediately. The library owns only its
- *    workspace (stream-ordered cudaMallocAsync on `stream`, or the caller's buffer via _ex).
- *    A is read-only.
+ *    workspace: stream-ordered allocations on `stream` from a memory pool the library creates for
+ *    the device (never the device's default pool; freed blocks stay cached in that pool until
+ *    wcsvd_trim_workspace), or the caller's buffer via _ex. The working copies W, V of Level >= 1
+ *    matrices (and the Level-0 park buffers) come from slot pools sized to the CTAs that can be
+ *    resident at once, not to the batch. A is read-only.
  *  - Asynchronous on `stream`: a return of WCSVD_OK means the work was enqueued.
  *  - Errors: negative codes are returned synchronously and nothing is enqueued on failure:
  *      -i          the i-th argument (1-based) is invalid (LAPACK convention);
@@ -27,7 +30,8 @@
  *  - Deterministic: the outputs for one matrix depend only on (m, n, the bits of A, tol,
  *    max_sweeps) -- never on batch composition, stream, device index or device count. The plan is
  *    a function of (m, n) only; there are no floating-point atomics.
- *  - Reentrant; no global mutable state.
+ *  - Reentrant. Process-wide state: only the per-device workspace pool above (created once, guarded
+ *    by a mutex); nothing a call does changes another call's results.
  */
 #ifndef WCSVD_H_
 #define WCSVD_H_
@@ -98,10 +102,12 @@ typedef struct {
                               Gram path, Level 2 of the W-cycle path) */
   int wcycle_sweeps;       /* 0 = planner (2); cap on Level-2 sweeps per W-cycle super-pair */
   int inner_sweeps;        /* 0 = planner (1); cap on EVD sweeps per pair */
-  int pair_warps;          /* 0 = planner (1); 2 = two warps per column-block pair on the flat Gram
-                              path with w = 16 (ablation, SURVEY §8(f2) lanes-per-pair; results are
-                              as deterministic, but not bitwise equal to the 1-warp executor: the
-                              Gram partials are summed in another order) */
+  int pair_warps;          /* 0 or 1: warps per column-block pair (the two-warp ablation executor of
+                              round 1 was removed; any other value is -12) */
+  int cluster_ctas;        /* 0 = planner (tailoring: a Gram-path matrix whose one-CTA time would
+                              dominate the batch is spread over a thread-block cluster of 2, 4 or 8
+                              CTAs); 1, 2, 4, 8 force the CTAs per Gram-path matrix (ablations).
+                              Results are bitwise independent of it. Other values: -12 */
 } wcsvd_opts;
 
 WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
@@ -128,21 +134,30 @@ WCSVD_API int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const 
  *     calling thread per chunk and overlap less).
  *   U, V: NULL, or an array of non-NULL pointers for every matrix (-7 if some entries are NULL).
  *   opts: as wcsvd_batched_ex, except that opts->info is a HOST int[batch]; workspace is ignored.
- * Pipeline: a uniform batch is cut into contiguous chunks (~500 matrices for Level 0, 8 for the Gram path); chunk c
- * is copied in (stream 1), factored on one of two compute streams, and copied out (stream 2) while chunk
- * c+1 is being copied in / factored, through two device staging sets (stream-ordered allocation). A mixed-size batch is one chunk
- * (its size buckets overlap each other instead). Host blocks of consecutive matrices that are adjacent
- * and packed (ld = rows) move as one copy (per matrix if the runtime refuses a merged range).
+ * Pipeline: the batch is cut into contiguous chunks of about equal estimated cost -- a uniform Level-0
+ * batch into ~500-matrix chunks (<= 32), a uniform Gram-path batch into min(16, batch / 128) chunks (at
+ * least 1), a mixed-size batch into 3 chunks when it has >= 300 matrices (else 1). Chunk c is copied in
+ * (stream 1), factored on one of two compute streams, and copied out (stream 2) while later chunks are
+ * copied in / factored, through three device staging sets (chunk c's H2D waits for the D2H of chunk
+ * c-3). Host blocks of consecutive matrices that are adjacent and packed (ld = rows) move as one copy
+ * (per matrix if the runtime refuses a merged range).
  * Ordered after prior work on `stream`; SYNCHRONOUS: returns when every output is in host memory.
  * Results are bitwise those of wcsvd_batched on the same inputs (per-matrix determinism).
- * Errors: the argument checks of wcsvd_batched (returned before anything is enqueued); ENOMEM if the
- * staging cannot be allocated; ECUDA on a failed copy or launch. */
+ * Errors: the argument checks of wcsvd_batched, opts fields and per-matrix plans included (returned
+ * before anything is allocated or enqueued); ENOMEM if the staging cannot be allocated; ECUDA on a
+ * failed copy or launch. */
 WCSVD_API int wcsvd_batched_host(int batch, const int* m, const int* n, const double* const* A, const int* lda,
                                  double* const* S, double* const* U, double* const* V, double tol,
                                  int max_sweeps, wcsvd_stream_t stream, const wcsvd_opts* opts);
 
-/* Bytes of device workspace wcsvd_batched_ex needs for this batch (host-only, no CUDA call). */
+/* Bytes of device workspace wcsvd_batched_ex needs for this batch with default options (planner
+ * tailoring; the slot pools are sized from the current device's SM count, 148 if no device is
+ * visible). 0 for an invalid batch. */
 WCSVD_API size_t wcsvd_workspace_size(int batch, const int* m, const int* n);
+
+/* Release the cached blocks of the library's workspace pool on the current device (after pending
+ * calls complete). Returns WCSVD_OK or WCSVD_ECUDA. */
+WCSVD_API int wcsvd_trim_workspace(void);
 
 /* Static string for a status code. */
 WCSVD_API const char* wcsvd_status_string(int status);

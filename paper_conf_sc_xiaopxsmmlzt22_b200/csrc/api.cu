@@ -9,6 +9,7 @@
 #include <cstdlib>
 #include <cstdint>
 #include <cstring>
+#include <mutex>
 #include <vector>
 
 #include "common.cuh"
@@ -92,56 +93,174 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   return WCSVD_OK;
 }
 
-size_t l1_bytes(const wcsvd_plan_t& p) {
-  if (p.path == WCSVD_PATH_L0) return (l0tp_park_bytes(p.variant, p.M) + 255) & ~size_t(255);
-  const size_t b = sizeof(double) * ((size_t)p.m_pad * p.n_pad + (size_t)p.n_pad * p.n_pad);
-  return (b + 255) & ~size_t(255);
+// Doubles of one workspace slot for a matrix with plan p: the Level >= 1 working copy W (m_pad x
+// n_pad) and V (n_pad x n_pad), or the Level-0 two-phase park buffer; 0 if the path needs none.
+size_t slot_doubles(const wcsvd_plan_t& p) {
+  if (p.path == WCSVD_PATH_L0) return ((l0tp_park_bytes(p.variant, p.M) + 255) & ~size_t(255)) / sizeof(double);
+  const size_t b = (size_t)p.m_pad * p.n_pad + (size_t)p.n_pad * p.n_pad;
+  return (b + 31) & ~size_t(31);
+}
+
+// Warps per CTA and resident CTAs per SM of the Level-1 variants (255 registers / thread, see
+// l1_gram.cu launch bounds): the tailoring rule and the slot-pool capacity use them.
+int l1_warps(int variant) { return variant == kL1_32x8 ? 8 : 4; }
+int resident_per_sm(const wcsvd_plan_t& p) {
+  if (p.path == WCSVD_PATH_L0) return 4;  // two-phase kernels: 128 registers, <= 4 CTAs per SM
+  return p.variant == kL1_32x8 ? 1 : 2;
+}
+
+int device_sms() {
+  int dev = 0, sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return 148;  // B200
+  }
+  return sms;
+}
+
+// Tailoring (PAPER.md:228 Challenge 2, §IV.D): CTAs per matrix for the
+// flat Gram path. A matrix whose one-CTA time would exceed the whole batch's ideal time on
+// the GPU (its cost share c_k / sum c > 1 / (R SMs)) is spread over a cluster of CL CTAs, the
+// smallest power of two that brings it under that bound, capped by the pair-level parallelism of a
+// round-robin step (ceil(pairs / warps); measured: 8 x 1024^2 in 903 / 455 / 234 / 233 ms on 1 / 2 /
+// 4 / 8 CTAs -- the dataflow schedule overlaps steps only a little) and 8.
+// A function of the batch's (m, n) multiset only -- it changes scheduling, never arithmetic (Z22).
+int choose_cluster(const wcsvd_plan_t& p, double share, int sms) {
+  if (p.path != WCSVD_PATH_GRAM) return 1;
+  const int nw = l1_warps(p.variant);
+  const int pairs = p.n_pad / p.w / 2;
+  int cap = 1;
+  while (cap < 8 && 2 * cap <= (pairs + nw - 1) / nw) cap *= 2;
+  static const double factor = [] {  // experiments only: WCSVD_TAILOR=<f> (default 1; measured C5 at 4 GPUs 776 / 812 / 840 ms for 1 / 2 / 4)
+    const char* s = std::getenv("WCSVD_TAILOR");
+    return s ? std::atof(s) : 1.0;
+  }();
+  const double need = factor * resident_per_sm(p) * sms * share;
+  int cl = 1;
+  while (cl < cap && cl < need) cl *= 2;
+  return cl;
 }
 
 struct Bucket {
-  int path, variant, withv;
+  int path, variant, withv, cluster;
   std::vector<int> members;  // batch indices, largest cost first
   int maxM = 0;
+  size_t slot = 0;  // doubles per slot (0: the path needs no workspace)
+  int nslots = 0;
+  size_t off_slots = 0, off_busy = 0;  // workspace offsets
 };
+
+// Plans, buckets and the workspace layout of one call: a pure function of (m, n, forced options,
+// which factors are requested) and of the device's SM count (slot-pool capacity only).
+struct CallPlan {
+  std::vector<wcsvd_plan_t> plans;
+  std::vector<Bucket> buckets;
+  size_t off_descs = 0, off_order = 0, off_status = 0, bytes = 0;
+};
+
+int make_call_plan(int batch, const int* m, const int* n, int force_path, int force_w, int force_cluster,
+                   const std::vector<int>* withv, CallPlan* cp) {
+  cp->plans.assign(batch, wcsvd_plan_t{});
+  double tot = 0;
+  for (int b = 0; b < batch; ++b) {
+    const int rc = plan_one(m[b], n[b], force_path, force_w, &cp->plans[b]);
+    if (rc != WCSVD_OK) return rc;
+    tot += cp->plans[b].cost;
+  }
+  const int sms = device_sms();
+  auto& buckets = cp->buckets;
+  buckets.clear();
+  for (int b = 0; b < batch; ++b) {
+    const wcsvd_plan_t& p = cp->plans[b];
+    int cl = force_cluster > 0 ? force_cluster : choose_cluster(p, tot > 0 ? p.cost / tot : 1.0, sms);
+    if (p.path != WCSVD_PATH_GRAM) cl = 1;
+    // the fused Level-0 kernel is instantiated per "V requested"; every other kernel reads d.withv
+    const bool fused_l0 = p.path == WCSVD_PATH_L0 && p.variant != kTP32 && p.variant != kTP64;
+    const int wv = (fused_l0 && withv) ? (*withv)[b] : 0;
+    Bucket* bk = nullptr;
+    for (auto& x : buckets)
+      if (x.path == p.path && x.variant == p.variant && x.withv == wv && x.cluster == cl) bk = &x;
+    if (!bk) {
+      buckets.push_back(Bucket{p.path, p.variant, wv, cl, {}, 0, 0, 0, 0, 0});
+      bk = &buckets.back();
+    }
+    bk->members.push_back(b);
+    bk->maxM = std::max(bk->maxM, p.M);
+    bk->slot = std::max(bk->slot, slot_doubles(p));
+  }
+  for (auto& bk : buckets)
+    std::stable_sort(bk.members.begin(), bk.members.end(),
+                     [&](int x, int y) { return cp->plans[x].cost > cp->plans[y].cost; });
+  std::sort(buckets.begin(), buckets.end(), [&](const Bucket& x, const Bucket& y) {
+    return cp->plans[x.members[0]].cost > cp->plans[y.members[0]].cost;
+  });
+  size_t off = 0;
+  auto align = [](size_t x) { return (x + 255) & ~size_t(255); };
+  cp->off_descs = off;
+  off = align(off + sizeof(MatDesc) * (size_t)batch);
+  cp->off_order = off;
+  off = align(off + sizeof(int) * (size_t)batch);
+  cp->off_status = off;
+  off = align(off + sizeof(int) * (size_t)batch);
+  for (auto& bk : buckets) {
+    if (!bk.slot) continue;
+    const int cap = std::max(1, (resident_per_sm(cp->plans[bk.members[0]]) * sms + bk.cluster - 1) / bk.cluster);
+    bk.nslots = std::min((int)bk.members.size(), cap);
+    if (std::getenv("WCSVD_SLOTS_ALL")) bk.nslots = (int)bk.members.size();  // experiments: one slot per matrix
+    bk.off_busy = off;
+    off = align(off + sizeof(int) * (size_t)bk.nslots);
+  }
+  for (auto& bk : buckets) {
+    if (!bk.slot) continue;
+    bk.off_slots = off;
+    off = align(off + sizeof(double) * bk.slot * (size_t)bk.nslots);
+  }
+  cp->bytes = off;
+  return WCSVD_OK;
+}
 
 const char* kStatus[] = {"ok", "invalid argument", "not supported", "CUDA error", "out of memory"};
 
-}  // namespace
-}  // namespace wcsvd
+// The library's own stream-ordered memory pool on `dev` (created once, kept for the process). Freed
+// workspace stays cached in it (release threshold = max) so repeated calls do not re-map memory; the
+// device's default pool and the caller's allocator are never touched. wcsvd_trim_workspace() releases it.
+std::mutex g_pool_mu;
+cudaMemPool_t g_pools[64] = {};
 
-using namespace wcsvd;
-
-static size_t ws_layout(int batch, const int* m, const int* n, size_t* off_descs, size_t* off_order,
-                        size_t* off_status, size_t* off_l1, std::vector<size_t>* l1_off = nullptr,
-                        int force_path = 0, int force_w = 0) {
-  size_t off = 0;
-  auto align = [](size_t x) { return (x + 255) & ~size_t(255); };
-  *off_descs = off;
-  off = align(off + sizeof(MatDesc) * (size_t)batch);
-  *off_order = off;
-  off = align(off + sizeof(int) * (size_t)batch);
-  *off_status = off;
-  off = align(off + sizeof(int) * (size_t)batch);
-  *off_l1 = off;
-  if (l1_off) l1_off->assign(batch, 0);
-  for (int b = 0; b < batch; ++b) {
-    wcsvd_plan_t p;
-    if (m[b] < 1 || n[b] < 1 || m[b] > kMaxDim || n[b] > kMaxDim) continue;
-    if (plan_one(m[b], n[b], force_path, force_w, &p) != WCSVD_OK) continue;
-    if (l1_off) (*l1_off)[b] = off;
-    off += l1_bytes(p);
+cudaError_t lib_pool(cudaMemPool_t* out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (!g_pools[dev]) {
+    cudaMemPoolProps props;
+    std::memset(&props, 0, sizeof(props));
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t p;
+    e = cudaMemPoolCreate(&p, &props);
+    if (e != cudaSuccess) return e;
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+    g_pools[dev] = p;
   }
-  return off;
+  *out = g_pools[dev];
+  return cudaSuccess;
 }
 
+cudaError_t lib_malloc(void** p, size_t bytes, cudaStream_t stream) {
+  cudaMemPool_t pool;
+  cudaError_t e = lib_pool(&pool);
+  if (e != cudaSuccess) return e;
+  return cudaMallocFromPoolAsync(p, bytes, pool, stream);
+}
+
+// Argument checks shared by every entry point (returned before anything is enqueued).
 template <typename TI>
-static int batched_impl(int batch, const int* m, const int* n, const TI* const* A, const int* lda,
-                        TI* const* S, TI* const* U, TI* const* V, double tol, int max_sweeps,
-                        wcsvd_stream_t stream_, const wcsvd_opts* opts) {
-  constexpr bool kF32 = sizeof(TI) == 4;
-  const double eps = kF32 ? 5.9604644775390625e-08 : kU53;  // 2^-24 or 2^-53
-  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
-  // ---- validation (nothing is enqueued on failure) ----
+int validate(int batch, const int* m, const int* n, const TI* const* A, const int* lda, TI* const* S, TI* const* U,
+             TI* const* V, double tol, const wcsvd_opts* opts) {
   if (batch < 0) return -1;
   if (batch == 0) return WCSVD_OK;
   if (!m) return -2;
@@ -164,76 +283,70 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
   }
   for (int b = 0; b < batch; ++b)
     if (m[b] > kMaxDim || n[b] > kMaxDim) return WCSVD_ENOTSUP;
+  if (opts) {
+    if (opts->pair_warps != 0 && opts->pair_warps != 1) return -12;
+    const int c = opts->cluster_ctas;
+    if (c != 0 && c != 1 && c != 2 && c != 4 && c != 8) return -12;
+    if (opts->force_path < 0 || opts->force_path > WCSVD_PATH_WCYCLE) return -12;
+    if (opts->force_w != 0 && opts->force_w != 8 && opts->force_w != 16) return -12;
+    for (int b = 0; b < batch; ++b) {
+      wcsvd_plan_t p;
+      const int rc = plan_one(m[b], n[b], opts->force_path, opts->force_w, &p);
+      if (rc != WCSVD_OK) return rc;
+    }
+  }
+  return WCSVD_OK;
+}
 
+}  // namespace
+}  // namespace wcsvd
+
+using namespace wcsvd;
+
+template <typename TI>
+static int batched_impl(int batch, const int* m, const int* n, const TI* const* A, const int* lda,
+                        TI* const* S, TI* const* U, TI* const* V, double tol, int max_sweeps,
+                        wcsvd_stream_t stream_, const wcsvd_opts* opts) {
+  constexpr bool kF32 = sizeof(TI) == 4;
+  const double eps = kF32 ? 5.9604644775390625e-08 : kU53;  // 2^-24 or 2^-53
+  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
+  // ---- validation (nothing is enqueued on failure) ----
+  const int vr = validate<TI>(batch, m, n, A, lda, S, U, V, tol, opts);
+  if (vr != WCSVD_OK || batch == 0) return vr;
+  const int* ldu = opts ? opts->ldu : nullptr;
+  const int* ldv = opts ? opts->ldv : nullptr;
   const int force_path = opts ? opts->force_path : 0;
   const int force_w = opts ? opts->force_w : 0;
   if (max_sweeps <= 0) max_sweeps = 60;
 
-  // ---- plan (a pure function of (m, n)) and bucket by kernel ----
-  std::vector<wcsvd_plan_t> plans(batch);
-  for (int b = 0; b < batch; ++b) {
-    const int rc = plan_one(m[b], n[b], force_path, force_w, &plans[b]);
-    if (rc != WCSVD_OK) return rc;
-  }
-  // Ablation (wcsvd_opts.pair_warps = 2): the flat Gram path with 2w = 32 on the split executor
-  // (two warps per column-block pair, l1_gram.cu).
-  if (opts && opts->pair_warps == 2)
-    for (auto& p : plans)
-      if (p.path == WCSVD_PATH_GRAM && (p.variant == kL1_32x8 || p.variant == kL1_32x4))
-        p.variant = (p.variant == kL1_32x8) ? kL1S_32x16 : kL1S_32x8;
-  if (opts && opts->pair_warps != 0 && opts->pair_warps != 1 && opts->pair_warps != 2) return -12;
+  // ---- plan (a pure function of (m, n)), tailoring and buckets ----
   // V_x (the square factor) is accumulated only if it is requested: as V when m >= n, as U when
   // m < n (§8(f4) values / U-only mode otherwise; the iteration itself is unchanged).
   std::vector<int> withv(batch);
   for (int b = 0; b < batch; ++b)
-    withv[b] = plans[b].swapped ? (U && U[b] ? 1 : 0) : (V && V[b] ? 1 : 0);
-  std::vector<Bucket> buckets;
-  for (int b = 0; b < batch; ++b) {
-    Bucket* bk = nullptr;
-    for (auto& x : buckets)
-      if (x.path == plans[b].path && x.variant == plans[b].variant && x.withv == withv[b]) bk = &x;
-    if (!bk) {
-      buckets.push_back(Bucket{plans[b].path, plans[b].variant, withv[b], {}, 0});
-      bk = &buckets.back();
-    }
-    bk->members.push_back(b);
-    bk->maxM = std::max(bk->maxM, plans[b].M);
-  }
-  for (auto& bk : buckets)
-    std::stable_sort(bk.members.begin(), bk.members.end(),
-                     [&](int x, int y) { return plans[x].cost > plans[y].cost; });
-  std::sort(buckets.begin(), buckets.end(), [&](const Bucket& x, const Bucket& y) {
-    return plans[x.members[0]].cost > plans[y.members[0]].cost;
-  });
+    withv[b] = (m[b] < n[b]) ? (U && U[b] ? 1 : 0) : (V && V[b] ? 1 : 0);
+  CallPlan cp;
+  const int rc0 = make_call_plan(batch, m, n, force_path, force_w, opts ? opts->cluster_ctas : 0, &withv, &cp);
+  if (rc0 != WCSVD_OK) return rc0;
+  const auto& plans = cp.plans;
+  const auto& buckets = cp.buckets;
 
-  // ---- workspace ----
-  size_t off_descs, off_order, off_status, off_l1;
-  std::vector<size_t> l1_off;
-  const size_t ws_bytes =
-      ws_layout(batch, m, n, &off_descs, &off_order, &off_status, &off_l1, &l1_off, force_path, force_w);
+  // ---- workspace: descriptors, launch order, status, slot pools ----
   unsigned char* ws = nullptr;
   bool own_ws = false;
   if (opts && opts->workspace) {
-    if (opts->workspace_bytes < ws_bytes) return -12;
+    if (opts->workspace_bytes < cp.bytes) return -12;
     ws = static_cast<unsigned char*>(opts->workspace);
   } else {
-    // Stream-ordered allocation from the device's default pool. Keep freed blocks cached in the
-    // pool (release threshold = max) so repeated calls do not re-map gigabytes of workspace.
-    int dev = 0;
-    cudaMemPool_t pool;
-    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-      uint64_t thr = UINT64_MAX;
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-    if (cudaMallocAsync(reinterpret_cast<void**>(&ws), ws_bytes, stream) != cudaSuccess) {
+    if (lib_malloc(reinterpret_cast<void**>(&ws), cp.bytes, stream) != cudaSuccess) {
       cudaGetLastError();
       return WCSVD_ENOMEM;
     }
     own_ws = true;
   }
-  MatDesc* d_descs = reinterpret_cast<MatDesc*>(ws + off_descs);
-  int* d_order = reinterpret_cast<int*>(ws + off_order);
-  int* d_status = reinterpret_cast<int*>(ws + off_status);
+  MatDesc* d_descs = reinterpret_cast<MatDesc*>(ws + cp.off_descs);
+  int* d_order = reinterpret_cast<int*>(ws + cp.off_order);
+  int* d_status = reinterpret_cast<int*>(ws + cp.off_status);
 
   // ---- descriptors (host) -> device ----
   std::vector<MatDesc> h(batch);
@@ -268,29 +381,29 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     d.idx = b;
     d.status = d_status;
     d.withv = withv[b];
-    if (p.path != WCSVD_PATH_L0) {
-      d.W = reinterpret_cast<double*>(ws + l1_off[b]);
-      d.Vw = d.W + (size_t)p.m_pad * p.n_pad;
-    } else if (l1_bytes(p)) {
-      d.W = reinterpret_cast<double*>(ws + l1_off[b]);  // two-phase L0 park buffer
-    }
   }
   std::vector<int> h_order;
   h_order.reserve(batch);
   std::vector<int> bucket_off;
+  size_t busy_lo = cp.bytes, busy_hi = 0;
   for (auto& bk : buckets) {
     bucket_off.push_back((int)h_order.size());
     h_order.insert(h_order.end(), bk.members.begin(), bk.members.end());
+    if (bk.slot) {
+      busy_lo = std::min(busy_lo, bk.off_busy);
+      busy_hi = std::max(busy_hi, bk.off_busy + sizeof(int) * (size_t)bk.nslots);
+    }
   }
   cudaError_t e = cudaMemcpyAsync(d_descs, h.data(), sizeof(MatDesc) * batch, cudaMemcpyHostToDevice, stream);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d_order, h_order.data(), sizeof(int) * batch, cudaMemcpyHostToDevice, stream);
+  if (e == cudaSuccess && busy_hi > busy_lo) e = cudaMemsetAsync(ws + busy_lo, 0, busy_hi - busy_lo, stream);
 
   // ---- launches ----
   // One launch per plan bucket (largest first). With several buckets (mixed sizes) each runs on its
   // own stream forked from `stream` so small buckets fill the SMs that large ones leave idle; all
   // are joined back into `stream` before the completion pass. Per-matrix results do not depend on
-  // this concurrency (each CTA owns one matrix).
+  // this concurrency, on the slot a matrix gets, or on its CTA count.
   const int nbk = (int)buckets.size();
   std::vector<cudaStream_t> side(nbk > 1 ? nbk : 0, nullptr);
   std::vector<cudaEvent_t> done(side.size(), nullptr);
@@ -308,12 +421,16 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     const Bucket& bk = buckets[i];
     const int cnt = (int)bk.members.size();
     cudaStream_t st = (nbk > 1) ? side[i] : stream;
+    SlotPool pool{nullptr, 0, nullptr, 0};
+    if (bk.slot) pool = SlotPool{reinterpret_cast<double*>(ws + bk.off_slots), bk.slot,
+                                 reinterpret_cast<int*>(ws + bk.off_busy), bk.nslots};
     if (bk.path == WCSVD_PATH_L0 && (bk.variant == kTP32 || bk.variant == kTP64))
-      e = launch_l0tp(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
+      e = launch_l0tp(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, pool, st);
     else if (bk.path == WCSVD_PATH_L0)
       e = launch_l0(bk.variant, bk.withv, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
-      e = launch_l1(bk.variant, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, st);
+      e = launch_l1(bk.variant, bk.path == WCSVD_PATH_WCYCLE ? 1 : 0, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i],
+                    cnt, bk.cluster, pool, st);
     if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);
   }
   for (int i = 0; i < (int)side.size(); ++i) {
@@ -327,6 +444,7 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
   if (e == cudaSuccess) e = launch_complete(kF32 ? 1 : 0, d_descs, batch, stream);
   if (own_ws) cudaFreeAsync(ws, stream);
   if (e != cudaSuccess) {
+    if (std::getenv("WCSVD_DEBUG")) std::fprintf(stderr, "wcsvd: %s\n", cudaGetErrorString(e));
     cudaGetLastError();
     return WCSVD_ECUDA;
   }
@@ -414,27 +532,11 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
                              double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
                              wcsvd_stream_t stream_, const wcsvd_opts* opts) {
   cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
-  if (batch < 0) return -1;
-  if (batch == 0) return WCSVD_OK;
-  if (!m) return -2;
-  if (!n) return -3;
-  if (!A) return -4;
-  if (!lda) return -5;
-  if (!S) return -6;
-  if (opts && opts->struct_size != sizeof(wcsvd_opts)) return -12;
+  // every argument (opts fields and per-matrix plans included) is checked before anything is enqueued
+  const int vr = validate<double>(batch, m, n, A, lda, S, U, V, tol, opts);
+  if (vr != WCSVD_OK || batch == 0) return vr;
   const int* ldu = opts ? opts->ldu : nullptr;
   const int* ldv = opts ? opts->ldv : nullptr;
-  for (int b = 0; b < batch; ++b) {
-    if (m[b] < 1) return -2;
-    if (n[b] < 1) return -3;
-    if (!A[b]) return -4;
-    if (lda[b] < m[b]) return -5;
-    if (!S[b]) return -6;
-    if (ldu && U && U[b] && ldu[b] < m[b]) return -12;
-    if (ldv && V && V[b] && ldv[b] < n[b]) return -12;
-  }
-  for (int b = 0; b < batch; ++b)
-    if (m[b] > kMaxDim || n[b] > kMaxDim) return WCSVD_ENOTSUP;
   const bool wantU = U != nullptr, wantV = V != nullptr;
   for (int b = 0; b < batch && (wantU || wantV); ++b)
     if ((wantU && !U[b]) || (wantV && !V[b])) return -7;  // host API: a factor is requested for all or none
@@ -455,12 +557,14 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   // C4 8 / 16 chunks 9804 / 10634 -> Gram path 16 chunks
   // mixed batches: 3 equal-cost chunks when large (C5, three staging sets, r01i: 1/2/3/4/6 chunks -> e2e
   // 892/906/927/745/620 matrices/s; beyond 3 every chunk is bounded by its own largest matrices)
+  // Gram path: 16 chunks at C3 / C4 sizes, fewer for small batches (~128 matrices per chunk at least,
+  // so a chunk still fills the GPU; a small batch is one chunk).
   int nch = batch >= 300 ? 3 : 1;
   if (uniform) {
     wcsvd_plan_t p0;
     const bool l0 = plan_one(m[0], n[0], opts ? opts->force_path : 0, opts ? opts->force_w : 0, &p0) == WCSVD_OK &&
                     p0.path == WCSVD_PATH_L0;
-    const int want = l0 ? std::min(32, (batch + 499) / 500) : 16;
+    const int want = l0 ? std::min(32, (batch + 499) / 500) : std::min(16, std::max(1, batch / 128));
     nch = std::max(1, std::min(batch, want));
   }
   if (const char* env = std::getenv("WCSVD_HOST_CHUNKS")) nch = std::max(1, std::min(batch, std::atoi(env)));  // experiments
@@ -504,7 +608,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   if (const char* env = std::getenv("WCSVD_HOST_SETS")) NSET = std::max(2, std::min(kHostSets, std::atoi(env)));  // experiments
   NSET = std::min(NSET, std::max(2, C));
   double* dbuf = nullptr;
-  if (cudaMallocAsync(reinterpret_cast<void**>(&dbuf), NSET * setB, stream) != cudaSuccess) {
+  if (lib_malloc(reinterpret_cast<void**>(&dbuf), NSET * setB, stream) != cudaSuccess) {
     cudaGetLastError();
     return WCSVD_ENOMEM;
   }
@@ -597,6 +701,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
       o.wcycle_sweeps = opts->wcycle_sweeps;
       o.inner_sweeps = opts->inner_sweeps;
       o.pair_warps = opts->pair_warps;
+      o.cluster_ctas = opts->cluster_ctas;
     }
     rc = batched_impl<double>(cnt, m + b0, n + b0, pA.data(), ld_.data(), pS.data(), wantU ? pU.data() : nullptr,
                               wantV ? pV.data() : nullptr, tol, max_sweeps,
@@ -688,8 +793,25 @@ int wcsvd_round_robin(int np, int step, int* pairs) {
 
 size_t wcsvd_workspace_size(int batch, const int* m, const int* n) {
   if (batch <= 0 || !m || !n) return 0;
-  size_t a, b, c, d;
-  return ws_layout(batch, m, n, &a, &b, &c, &d);
+  for (int b = 0; b < batch; ++b)
+    if (m[b] < 1 || n[b] < 1 || m[b] > kMaxDim || n[b] > kMaxDim) return 0;
+  CallPlan cp;
+  if (make_call_plan(batch, m, n, 0, 0, 0, nullptr, &cp) != WCSVD_OK) return 0;
+  return cp.bytes;
+}
+
+int wcsvd_trim_workspace(void) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ECUDA;
+  }
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (dev >= 0 && dev < 64 && g_pools[dev] && cudaMemPoolTrimTo(g_pools[dev], 0) != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ECUDA;
+  }
+  return WCSVD_OK;
 }
 
 int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,

@@ -71,6 +71,31 @@ struct MatDesc {
   int* status;  // internal per-matrix status flags (workspace), e.g. kNeedsCompletion
 };
 
+// Workspace slot pool: the Level-1 working copies (W + V) and the Level-0 two-phase park buffers are
+// not allocated per matrix but per RESIDENT CTA (or cluster): a CTA takes a free slot when it starts
+// (atomicCAS on busy[]) and returns it when it exits. nslots is the bucket's resident capacity; if more
+// CTAs happen to be resident than slots exist, the extra ones wait -- never deadlocks, because slot
+// holders wait on nothing the waiters hold. Which slot a matrix gets changes no arithmetic.
+struct SlotPool {
+  double* base;         // nslots x slot_doubles
+  size_t slot_doubles;  // doubles per slot (the bucket's largest matrix)
+  int* busy;            // [nslots], zero before the launch
+  int nslots;
+};
+__device__ __forceinline__ int slot_acquire(const SlotPool& p, int hint) {
+  for (int i = hint % p.nslots, tries = 0;; i = (i + 1 == p.nslots) ? 0 : i + 1) {
+    if (atomicCAS(&p.busy[i], 0, 1) == 0) {
+      __threadfence();
+      return i;
+    }
+    if (++tries % p.nslots == 0) __nanosleep(256);  // every slot held: wait for an owner to finish
+  }
+}
+__device__ __forceinline__ void slot_release(const SlotPool& p, int s) {
+  __threadfence();
+  atomicExch(&p.busy[s], 0);
+}
+
 // Status flags a kernel can leave for the completion pass (Z14): bit 0 = some sigma_j below the
 // rank threshold; those U columns were written as 0 and need the deterministic MGS completion.
 constexpr int kNeedsCompletion = 1;

@@ -25,14 +25,15 @@ enum L1Variant {
   kL1_16x4 = 11,  // 2w = 16, 4 warps
   kL1_32x4 = 12,  // 2w = 32, 4 warps
   kL1_32x8 = 13,  // 2w = 32, 8 warps
-  kL1S_32x8 = 14,   // 2w = 32, split executor (2 warps per pair): 4 pair groups, 8 warps
-  kL1S_32x16 = 15,  // 2w = 32, split executor: 8 pair groups, 16 warps
 };
 
-cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream);
+// Level-1 launch: `cluster` CTAs per matrix (1, 2, 4 or 8; a thread-block cluster when > 1).
+// wcycle = 1: the W-cycle kernel (Level 1 -> Level 2 recursion, one CTA per matrix).
+cudaError_t launch_l1(int variant, int wcycle, int fp32, const MatDesc* descs, const int* order, int count,
+                      int cluster, const SlotPool& pool, cudaStream_t stream);
 
 cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
-                        cudaStream_t stream);
+                        const SlotPool& pool, cudaStream_t stream);
 size_t l0tp_park_bytes(int variant, int M);  // per-matrix park buffer (X and V_x registers), fp64
 
 cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, const int* order, int count,

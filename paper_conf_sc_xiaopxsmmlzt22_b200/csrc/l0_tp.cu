@@ -423,7 +423,7 @@ constexpr size_t l0tp_park_elems(int nt) {
 // gv = t % GV) holds row rv x slots gv*NP/GV .. of V_x.
 template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB, bool WL>
 __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restrict__ descs,
-                                                          const int* __restrict__ order) {
+                                                          const int* __restrict__ order, SlotPool pool) {
   static_assert(!WL || (!RED && RX == 4 && NP / GX == 8 && MAXT == 16 * GX), "warp-local layout");
   using V2 = typename Prec<T>::V2;
   constexpr int NLX = NP / GX;
@@ -456,8 +456,12 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
   int* s_rank = reinterpret_cast<int*>(s_sgn + NP);                       // [NP]
   int* s_flags = s_rank + NP;                                             // [8]
   T* s_vbest = reinterpret_cast<T*>(s_rot);  // finalisation: [RW4][NP] sign-rule scratch (aliases s_rot)
+  __shared__ int s_slot;  // park-buffer slot of this CTA (SlotPool: sized to resident CTAs, not the batch)
   if (tid < 8) s_flags[tid] = 0;
-  if (tid == 0) *s_max = 0ull;
+  if (tid == 0) {
+    *s_max = 0ull;
+    s_slot = slot_acquire(pool, blockIdx.x);
+  }
   for (int e = tid; e < (RED ? 6 : 3) * RW4 * PS; e += NT) s_part[e] = T(0);
   __syncthreads();
 
@@ -516,7 +520,7 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
   cx.tol2 = (T)(d.tol * d.tol);
   cx.par = 0;
   cx.nwarp = NT / 32;
-  T* parkX = reinterpret_cast<T*>(d.W);
+  T* parkX = reinterpret_cast<T*>(pool.base + (size_t)s_slot * pool.slot_doubles);
   T* parkV = parkX + (size_t)NT * RX * NLX;
   int sweep = 0;
   bool converged = false;
@@ -691,6 +695,7 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
     if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
     if (d.sweeps_inner) d.sweeps_inner[d.idx] = 0;
     if (d.status) d.status[d.idx] = (s_flags[3] && dstW) ? kNeedsCompletion : 0;
+    slot_release(pool, s_slot);
   }
 }
 
@@ -702,14 +707,15 @@ constexpr int tp_threads(int M) {
 }
 
 template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB, bool WL>
-static cudaError_t launch_tp_t(const MatDesc* descs, const int* order, int count, int maxM, cudaStream_t stream) {
+static cudaError_t launch_tp_t(const MatDesc* descs, const int* order, int count, int maxM, const SlotPool& pool,
+                               cudaStream_t stream) {
   const int threads = tp_threads<NP, GX, RX, GV>(maxM);
   if (threads > MAXT) return cudaErrorInvalidConfiguration;
   const size_t smem = l0tp_smem_bytes<T, NP, GX, RX, RED>(maxM, threads);
   auto kern = l0tp_kernel<T, NP, GX, RX, GV, RED, MAXT, MINB, WL>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  kern<<<count, threads, smem, stream>>>(descs, order);
+  kern<<<count, threads, smem, stream>>>(descs, order, pool);
   return cudaGetLastError();
 }
 
@@ -785,20 +791,22 @@ int l0tp_occupancy(int variant, int fp32, int maxM) {
 }
 
 template <typename T, int V>
-static cudaError_t launch_v(const MatDesc* descs, const int* order, int count, int maxM, cudaStream_t stream) {
+static cudaError_t launch_v(const MatDesc* descs, const int* order, int count, int maxM, const SlotPool& pool,
+                            cudaStream_t stream) {
   using C = TPCfg<V>;
-  return launch_tp_t<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB, C::WL>(descs, order, count, maxM, stream);
+  return launch_tp_t<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB, C::WL>(descs, order, count, maxM, pool,
+                                                                                    stream);
 }
 
 cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
-                        cudaStream_t stream) {
+                        const SlotPool& pool, cudaStream_t stream) {
   switch (variant) {
     case kTP32:
-      return fp32 ? launch_v<float, kTP32>(descs, order, count, maxM, stream)
-                  : launch_v<double, kTP32>(descs, order, count, maxM, stream);
+      return fp32 ? launch_v<float, kTP32>(descs, order, count, maxM, pool, stream)
+                  : launch_v<double, kTP32>(descs, order, count, maxM, pool, stream);
     case kTP64:
-      return fp32 ? launch_v<float, kTP64>(descs, order, count, maxM, stream)
-                  : launch_v<double, kTP64>(descs, order, count, maxM, stream);
+      return fp32 ? launch_v<float, kTP64>(descs, order, count, maxM, pool, stream)
+                  : launch_v<double, kTP64>(descs, order, count, maxM, pool, stream);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -281,61 +281,6 @@ __device__ __forceinline__ void store_sym(double* buf, const double (&acc)[PairC
       }
 }
 
-// X (rows x 2w panel of columns pcol(.), leading dim ld) <- X * J', J' given as B fragments
-// jf[kk][nb] = J'[4kk + l%4][8nb + l/4]. In place, 16-row slabs; the next slab's A fragments are
-// loaded while the current slab is multiplied (register ping-pong).
-template <int W2>
-__device__ __forceinline__ void rot_load(double (&a)[2][W2 / 4], const double* base, const int (&oa)[W2 / 4],
-                                         int r0) {
-#pragma unroll
-  for (int h = 0; h < 2; ++h)
-#pragma unroll
-    for (int kk = 0; kk < W2 / 4; ++kk) a[h][kk] = base[oa[kk] + r0 + 8 * h];
-}
-
-template <int W2>
-__device__ __forceinline__ void rot_mma_store(const double (&a)[2][W2 / 4], const double (&jf)[W2 / 4][W2 / 8],
-                                              double* base, const int (&oc)[W2 / 8][2], int r0) {
-  constexpr int CG = W2 / 8, KK = W2 / 4;
-#pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    double acc[CG][2];
-#pragma unroll
-    for (int nb = 0; nb < CG; ++nb) acc[nb][0] = acc[nb][1] = 0.0;
-#pragma unroll
-    for (int kk = 0; kk < KK; ++kk)
-#pragma unroll
-      for (int nb = 0; nb < CG; ++nb) dmma884(acc[nb], a[h][kk], jf[kk][nb]);
-#pragma unroll
-    for (int nb = 0; nb < CG; ++nb)
-#pragma unroll
-      for (int e = 0; e < 2; ++e) base[oc[nb][e] + r0 + 8 * h] = acc[nb][e];
-  }
-}
-
-template <int W2>
-__device__ __forceinline__ void apply_rotation(double* base, int ld, int rows, int I, int J, int lane,
-                                               const double (&jf)[W2 / 4][W2 / 8]) {
-  constexpr int CG = W2 / 8, KK = W2 / 4;
-  int oa[KK], oc[CG][2];  // element offsets (a panel is < 2^31 elements)
-#pragma unroll
-  for (int kk = 0; kk < KK; ++kk) oa[kk] = pcol<W2>(4 * kk + (lane & 3), I, J) * ld + (lane >> 2);
-#pragma unroll
-  for (int nb = 0; nb < CG; ++nb)
-#pragma unroll
-    for (int e = 0; e < 2; ++e) oc[nb][e] = pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
-  double a0[2][KK], a1[2][KK];
-  rot_load<W2>(a0, base, oa, 0);
-  for (int r0 = 0;;) {
-    if (r0 + 16 < rows) rot_load<W2>(a1, base, oa, r0 + 16);
-    rot_mma_store<W2>(a0, jf, base, oc, r0);
-    if ((r0 += 16) >= rows) break;
-    if (r0 + 16 < rows) rot_load<W2>(a0, base, oa, r0 + 16);
-    rot_mma_store<W2>(a1, jf, base, oc, r0);
-    if ((r0 += 16) >= rows) break;
-  }
-}
-
 // ---- Inner EVD storage: B in "slot" order, moved along with the round-robin ring ----
 // B (symmetric, 2w x 2w) is kept as its upper triangle indexed by *slot*: the pair k of every step
 // is always slots (2k, 2k+1), so the elements a lane reads (its 2x2 quads) sit at the same
@@ -601,405 +546,101 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(5);
   return true;
 }
-
-// ---- Split pair executor: two warps per column-block pair (2w = 32) ----
-// The EVD of one pair is issue- and latency-bound in a single warp (~600 instructions and a
-// sqrt/rsqrt chain per step, tools/evd_probe.cu), so a pair is owned by a group of two warps:
-// warp h of the group computes the Gram partial and the A / V update over its half of the rows,
-// holds the J columns of slot half h (slots 16h .. 16h+15, lane = row of J), and updates its half
-// of the off-diagonal quads of B (64-lane EvdMap). Both warps evaluate every rotation of a step
-// (bitwise the same numbers); warp 0 writes the diagonal blocks. One named barrier per EVD step
-// publishes B' and the two J values that cross between the column halves (the circle-method ring
-// moves slot 14 -> 16 and slot 17 -> 15, common.cuh). Twice the warps per SM at the same on-chip
-// footprint per matrix.
-constexpr int kSplitW2 = 32;
-constexpr int kSplitNS = 2;       // slab-ring stages per warp
-constexpr int kSplitSlab = 32 * 16;  // doubles per slab: 32 columns x 16 rows, XOR-swizzled rows (no pad)
-
-struct SplitSmem {
-  double* B;     // [2][W2 * W2] EVD ping-pong (slot layout); afterwards E = J^T J - I (stride BS)
-  double* S;     // [W2][BS] staged J
-  double* jf;    // [W2/4][W2/8][32] J' as DMMA B fragments (aliases S; written once S is consumed)
-  double* ring;  // this warp's [kSplitNS][kSplitSlab] slab ring (aliases B)
-  double* red;   // [NTU][2][32] Gram partials of warp 1 (inside warp 1's ring)
-  double2* cs;   // this warp's [W2 / 2] (c, s) of the current step
-  double* xch;   // [2 parity][2 halves][32] J values crossing between the column halves
-  // doubles: B [0, 2048), S [2048, 2048 + 32 * 33), jf [2048, 3072), rings [0, 2 * NS * slab)
-  __host__ __device__ static constexpr size_t region() {
-    constexpr size_t evd = (size_t)2 * kSplitW2 * kSplitW2 + (size_t)kSplitW2 * PairCfg<kSplitW2>::BS;
-    constexpr size_t rings = (size_t)2 * kSplitNS * kSplitSlab;
-    static_assert(rings <= 2 * kSplitW2 * kSplitW2, "rings must not reach the J' fragments");
-    return (evd > rings ? evd : rings) * sizeof(double);
-  }
-  __host__ __device__ static constexpr size_t bytes() {  // per group
-    return region() + 2 * sizeof(double2) * (kSplitW2 / 2) + sizeof(double) * 2 * 2 * 32;
-  }
-};
-
-// J columns of slot half HC: the value of global slot `gs` after the step goes to its next slot
-// (common.cuh rr_dest); within the half it is a register rename, across the halves it is sent.
-template <int HC>
-__device__ __forceinline__ void split_place(int gs, double v, double (&y)[16], double& send) {
-  const int dst = rr_dest(gs, kSplitW2) - 16 * HC;
-  if (dst >= 0 && dst < 16) y[dst] = v;
-  else send = v;
+// ---- Cross-CTA plumbing for a matrix spread over a thread-block cluster (tailoring) ----
+// A matrix may be owned by a cluster of CL CTAs (CL = 1, 2, 4, 8; chosen by the planner from the batch
+// composition, PAPER.md:228, 261-269 -- scheduling only, never arithmetic, Z22). The pairs of a
+// round-robin step are spread over all CL x NW warps of the cluster; the per-block dataflow counters,
+// the convergence vote and the finalisation arrays live in the shared memory of CTA rank 0 and are
+// reached through distributed shared memory (generic addresses from map_shared_rank). W and V stay in
+// the global (L2-resident) slot of the matrix; every pair's arithmetic is that of the one-CTA kernel,
+// so results are bitwise independent of CL (tests/test_gpu_cluster.py).
+__device__ __forceinline__ unsigned cl_rank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
 }
-
-template <int HC>
-__device__ __forceinline__ bool evd_step_split(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
-                                               const EvdMap<kSplitW2, 64>& em, int lane, double tol2,
-                                               const double (&x)[16], double (&y)[16], double& send) {
-  constexpr int W2 = kSplitW2, NPR = W2 / 2, QPL = EvdMap<W2, 64>::QPL;
-  const double bpp = Bc[em.dld01 & 0xffff], bqq = Bc[em.dld01 >> 16], bpq = Bc[em.dld2];
-  double c, s, t;
-  const bool rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
-  if (lane < NPR) {
-    cs[lane] = make_double2(c, s);
-    if (HC == 0) {
-      Bn[em.dst01 & 0xffff] = rot ? fma(t, bpq, bpp) : bpp;
-      Bn[em.dst01 >> 16] = rot ? fma(-t, bpq, bqq) : bqq;
-      Bn[em.dst2] = rot ? 0.0 : bpq;
-    }
-  }
-  double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
-#pragma unroll
-  for (int i = 0; i < QPL; ++i) {
-    if (em.q[i] & (1 << 13)) {
-      const int o = em.q[i] & 0x7ff;
-      const double2 v0 = *reinterpret_cast<const double2*>(Bc + o);
-      const double2 v1 = *reinterpret_cast<const double2*>(Bc + o + W2);
-      const bool sw = (em.q[i] >> 11) & 1;
-      b00[i] = sw ? v0.y : v0.x;
-      b01[i] = sw ? v0.x : v0.y;
-      b10[i] = sw ? v1.y : v1.x;
-      b11[i] = sw ? v1.x : v1.y;
-    }
-  }
-  if (!__any_sync(0xffffffffu, rot)) {
-#pragma unroll
-    for (int i = 0; i < QPL; ++i) {
-      if (em.q[i] & (1 << 13)) {
-        Bn[em.st[i][0] & 0xffff] = b00[i];
-        Bn[em.st[i][0] >> 16] = b01[i];
-        Bn[em.st[i][1] & 0xffff] = b10[i];
-        Bn[em.st[i][1] >> 16] = b11[i];
-      }
-    }
-#pragma unroll
-    for (int j = 0; j < 16; ++j) split_place<HC>(16 * HC + j, x[j], y, send);
-    return false;
-  }
-  __syncwarp();
-#pragma unroll
-  for (int i = 0; i < QPL; ++i) {
-    if (em.q[i] & (1 << 13)) {
-      const double2 gp = cs[(em.q[i] >> 16) & (NPR - 1)];
-      const bool own_lo = (em.q[i] >> 12) & 1;
-      const double rc = own_lo ? c : gp.x, rs = own_lo ? s : gp.y;
-      const double cc = own_lo ? gp.x : c, cs_ = own_lo ? gp.y : s;
-      const double c0 = fma(cs_, b01[i], cc * b00[i]), c1 = fma(-cs_, b00[i], cc * b01[i]);
-      const double d0 = fma(cs_, b11[i], cc * b10[i]), d1 = fma(-cs_, b10[i], cc * b11[i]);
-      Bn[em.st[i][0] & 0xffff] = fma(rs, d0, rc * c0);
-      Bn[em.st[i][0] >> 16] = fma(rs, d1, rc * c1);
-      Bn[em.st[i][1] & 0xffff] = fma(-rs, c0, rc * d0);
-      Bn[em.st[i][1] >> 16] = fma(-rs, c1, rc * d1);
-    }
-  }
-#pragma unroll
-  for (int kk = 0; kk < 8; ++kk) {
-    const double2 g = cs[8 * HC + kk];
-    const double a = x[2 * kk], b = x[2 * kk + 1];
-    split_place<HC>(16 * HC + 2 * kk, fma(g.y, b, g.x * a), y, send);
-    split_place<HC>(16 * HC + 2 * kk + 1, fma(-g.y, a, g.x * b), y, send);
-  }
-  return true;
+__device__ __forceinline__ unsigned cl_nrank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+  return r;
 }
-
-// Split-executor panel streaming (2w = 32): the slab ring of gram_tiles_async / apply_rotation_async
-// with 16-double columns and the rows of column c stored XOR (4 (c mod 4)) (conflict-free fragment
-// reads without padding), panel addresses formed from the two block bases, and J' read from shared
-// memory (fragment order) instead of registers -- the executor runs at 128 registers per thread.
-__device__ __forceinline__ int slab_at(int c, int r) { return c * 16 + (r ^ (4 * (c & 3))); }
-
-struct SplitPanel {
-  const double* gI;  // this lane's copy source in block I: column I*16 + lane/8, rows 2 (lane%8) + {0,1}
-  const double* gJ;
-  size_t ld4;        // 4 columns
-  int so;            // this lane's slab offset of (column lane/8, rows 2 (lane%8)); + 64 i for column + 4 i
-  __device__ __forceinline__ SplitPanel(const double* base, int ld, int I, int J, int lane) {
-    gI = base + (size_t)(I * 16 + (lane >> 3)) * ld + 2 * (lane & 7);
-    gJ = base + (size_t)(J * 16 + (lane >> 3)) * ld + 2 * (lane & 7);
-    ld4 = (size_t)4 * ld;
-    so = slab_at(lane >> 3, 2 * (lane & 7));  // column lane/8 + 4 i has the same swizzle
-  }
-  __device__ __forceinline__ void issue(double* ring, int r0, int st) const {
-    double* dst = ring + st * kSplitSlab + so;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) cp_async16(dst + 64 * i, (i < 4 ? gI : gJ) + (i & 3) * ld4 + r0);
-  }
-};
-
-__device__ __forceinline__ void gram_split(double* ring, const double* base, int ld, int rows, int I, int J, int lane,
-                                           double (&acc)[PairCfg<kSplitW2>::NTU][2]) {
-  constexpr int W2 = kSplitW2, CG = W2 / 8, NS = kSplitNS;
-#pragma unroll
-  for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
-  const SplitPanel pn(base, ld, I, J, lane);
-  const int nslab = rows >> 4;
-#pragma unroll
-  for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) pn.issue(ring, 16 * j, j);
-    cp_async_commit();
-  }
-  // fragment (column 8 c + lane/4, row lane%4 + 4 u)
-  const int fc = (lane >> 2) * 16, fr = lane & 3, fx = (lane >> 2) & 3;
-  for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) pn.issue(ring, 16 * (sl + NS - 1), (sl + NS - 1) % NS);
-    cp_async_commit();
-    cp_async_wait<NS - 1>();
-    __syncwarp();
-    const double* st = ring + (sl % NS) * kSplitSlab + fc + fr;
-    double f[4][CG];
-#pragma unroll
-    for (int u = 0; u < 4; ++u)
-#pragma unroll
-      for (int c = 0; c < CG; ++c) f[u][c] = st[128 * c + 4 * (u ^ fx)];
-    gram_mma<W2>(acc, f);
-    __syncwarp();
+__device__ __forceinline__ unsigned cl_id() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r));
+  return r;
+}
+// Cluster-wide barrier with release / acquire semantics (orders global and shared memory).
+__device__ __forceinline__ void cl_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// Generic address of `p` (a __shared__ variable) in the CTA of cluster rank 0.
+template <typename T>
+__device__ __forceinline__ T* at_rank0(T* p) {
+  uint64_t g;
+  asm volatile("mapa.u64 %0, %1, 0;" : "=l"(g) : "l"(reinterpret_cast<uint64_t>(p)));
+  return reinterpret_cast<T*>(g);
+}
+// Dataflow counter of a column block: acquire-load / release-store at CTA scope (one CTA per matrix)
+// or at cluster scope (the counter sits in rank 0's shared memory).
+template <bool CLU>
+__device__ __forceinline__ int ver_acquire(int* p) {
+  if constexpr (CLU) {
+    int v;
+    asm volatile("ld.acquire.cluster.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+  } else {
+    return atomicAdd(p, 0);  // relaxed read; the fence after the spin orders the panel reads
   }
 }
-
-__device__ __forceinline__ void apply_split(double* ring, double* base, int ld, int rows, int I, int J, int lane,
-                                            const double* __restrict__ jfs) {
-  constexpr int W2 = kSplitW2, CG = W2 / 8, KK = W2 / 4, NS = kSplitNS;
-  const SplitPanel pn(base, ld, I, J, lane);
-  // output element (row 16 sl + 8 h + lane/4, panel column 8 nb + 2 (lane%4) + e)
-  double* oI = base + (size_t)(I * 16 + 2 * (lane & 3)) * ld + (lane >> 2);
-  double* oJ = base + (size_t)(J * 16 + 2 * (lane & 3)) * ld + (lane >> 2);
-  const int nslab = rows >> 4;
-#pragma unroll
-  for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) pn.issue(ring, 16 * j, j);
-    cp_async_commit();
-  }
-  // A fragment (row 8 h + lane/4, column 4 kk + lane%4)
-  const int fa0 = slab_at(lane & 3, lane >> 2), fa1 = slab_at(lane & 3, 8 + (lane >> 2));
-  const double* jl = jfs + lane;
-  for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) pn.issue(ring, 16 * (sl + NS - 1), (sl + NS - 1) % NS);
-    cp_async_commit();
-    cp_async_wait<NS - 1>();
-    __syncwarp();
-    const double* st = ring + (sl % NS) * kSplitSlab;
-    double acc0[CG][2], acc1[CG][2];
-#pragma unroll
-    for (int nb = 0; nb < CG; ++nb) acc0[nb][0] = acc0[nb][1] = acc1[nb][0] = acc1[nb][1] = 0.0;
-#pragma unroll
-    for (int kk = 0; kk < KK; ++kk) {
-      const double a0 = st[64 * kk + fa0], a1 = st[64 * kk + fa1];
-#pragma unroll
-      for (int nb = 0; nb < CG; ++nb) {
-        const double bj = jl[(kk * CG + nb) * 32];
-        dmma884(acc0[nb], a0, bj);
-        dmma884(acc1[nb], a1, bj);
-      }
-    }
-#pragma unroll
-    for (int nb = 0; nb < CG; ++nb)
-#pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        double* o = (nb < 2 ? oI : oJ) + (size_t)(8 * (nb & 1) + e) * ld + 16 * sl;
-        __stcg(o, acc0[nb][e]);
-        __stcg(o + 8, acc1[nb][e]);
-      }
-    __syncwarp();
-  }
+template <bool CLU>
+__device__ __forceinline__ void ver_release(int* p, int v) {
+  if constexpr (CLU)
+    asm volatile("st.release.cluster.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  else
+    atomicExch(p, v);
+}
+template <bool CLU>
+__device__ __forceinline__ void pair_fence() {
+  if constexpr (CLU)
+    __threadfence();  // the panels of the pair are read / written by warps on other SMs
+  else
+    __threadfence_block();
 }
 
-// Rows [0, h) go to warp 0 and [h, rows) to warp 1, h a multiple of 16.
-__device__ __forceinline__ int split_rows(int rows) { return 16 * (((rows >> 4) + 1) >> 1); }
-
-// One column-block pair (I, J) by the group's warp HC (bar_id: the group's named barrier).
-template <int HC>
-__device__ bool process_pair_split(const SplitSmem& ss, double* Wm, int ld, int mrows, double* Vm, int ldv,
-                                   int vrows, int I, int J, double tol2, int inner_cap, int lane, int bar_id,
-                                   int* inner) {
-  constexpr int W2 = kSplitW2;
-  using C = PairCfg<W2>;
-  constexpr int CG = C::CG, BS = C::BS, NTU = C::NTU;
-  double* B0 = ss.B;
-  double* B1 = ss.B + W2 * W2;
-  const int hm = split_rows(mrows);
-  const int r0 = HC ? hm : 0, nr = HC ? mrows - hm : hm;
-  PHASE_T0();
-  // (1) Gram B = P^T P (Alg 1 l.5): partials over each warp's rows, summed in a fixed order.
-  {
-    double acc[NTU][2];
-    gram_split(ss.ring, Wm + r0, ld, nr, I, J, lane, acc);
-    if (HC == 1) {
-#pragma unroll
-      for (int t = 0; t < NTU; ++t)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) ss.red[(2 * t + e) * 32 + lane] = acc[t][e];
-    }
-    named_bar(bar_id, 64);
-    if (HC == 0) {
-      int t = 0;
-#pragma unroll
-      for (int a = 0; a < CG; ++a)
-#pragma unroll
-        for (int b = a; b < CG; ++b, ++t)
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const int row = 8 * a + (lane >> 2), col = 8 * b + 2 * (lane & 3) + e;
-            const double v = acc[t][e] + ss.red[(2 * t + e) * 32 + lane];
-            if (a != b || row <= col) B0[evd_phys<W2>(row, col)] = v;
-          }
-    }
-    named_bar(bar_id, 64);
-  }
-  PHASE_MARK(0);
-  // (4) off-norm test (Z6), evaluated identically by both warps.
-  bool need = false;
-  {
-    const double bqq = B0[evd_phys<W2>(lane, lane)];
-#pragma unroll 4
-    for (int p = 0; p < W2 - 1; ++p) {
-      const double bpp = B0[evd_phys<W2>(p, p)];
-      const double bpq = (lane > p) ? B0[evd_phys<W2>(p, lane)] : 0.0;
-      const double ab = bpp * bqq;
-      need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
-    }
-  }
-  PHASE_MARK(1);
-  PHASE_COUNT(7);
-  if (!__any_sync(0xffffffffu, need)) return false;
-  // (2) EVD of B (Alg 1 l.6), threshold parallel Jacobi split over the group.
-  EvdMap<W2, 64> em;
-  em.init(32 * HC + lane);
-  double ja[16], jb[16];
-#pragma unroll
-  for (int s = 0; s < 16; ++s) ja[s] = (lane == 16 * HC + s) ? 1.0 : 0.0;
-  constexpr int RECV = HC ? 0 : 15;  // local slot that receives the crossing value
-  double* xo = ss.xch + HC * 32 + lane;        // + parity * 64
-  const double* xi = ss.xch + (HC ^ 1) * 32 + lane;
-  int par = 0;
-  bool rotated = false;
-  int isw = 0;
-  for (; isw < inner_cap; ++isw) {
-    double send = 0.0;
-    bool any = evd_step_split<HC>(B0, B1, ss.cs, em, lane, tol2, ja, jb, send);
-    xo[par * 64] = send;
-    named_bar(bar_id, 64);
-    jb[RECV] = xi[par * 64];
-    par ^= 1;
-    for (int r = 1; r < W2 - 1; r += 2) {
-      any |= evd_step_split<HC>(B1, B0, ss.cs, em, lane, tol2, jb, ja, send);
-      xo[par * 64] = send;
-      named_bar(bar_id, 64);
-      ja[RECV] = xi[par * 64];
-      par ^= 1;
-      any |= evd_step_split<HC>(B0, B1, ss.cs, em, lane, tol2, ja, jb, send);
-      xo[par * 64] = send;
-      named_bar(bar_id, 64);
-      jb[RECV] = xi[par * 64];
-      par ^= 1;
-    }
-#pragma unroll
-    for (int s = 0; s < 16; ++s) ja[s] = jb[s];
-    double* tmp = B0;
-    B0 = B1;
-    B1 = tmp;
-    rotated |= any;
-    if (!any) break;
-  }
-  if (HC == 0) *inner += isw + (isw < inner_cap ? 1 : 0);
-  PHASE_MARK(2);
-  PHASE_COUNT(6);
-  if (!rotated) return false;
-  // Newton-Schulz (Z9(ii)): E = J^T J - I (warp 0), J' = J - J E / 2 (rows 16 HC .. 16 HC + 15).
-#pragma unroll
-  for (int s = 0; s < 16; ++s) ss.S[lane * BS + 16 * HC + s] = ja[s];
-  named_bar(bar_id, 64);
-  if (HC == 0) {
-    const double* ptr[CG];
-#pragma unroll
-    for (int c = 0; c < CG; ++c) ptr[c] = ss.S + (lane & 3) * BS + 8 * c + (lane >> 2);
-    double acc[NTU][2];
-    gram_tiles<W2>(ptr, W2, BS, acc);
-    store_sym<W2>(ss.B, acc, lane, 1.0);
-  }
-  named_bar(bar_id, 64);
-  {
-    double jn[2][CG][2];  // rows 8 (2 HC + ii) + lane/4 of J', columns 8 j + 2 (lane%4) + e
-#pragma unroll
-    for (int ii = 0; ii < 2; ++ii)
-#pragma unroll
-      for (int j = 0; j < CG; ++j) {
-        const int i = 2 * HC + ii;
-        double acc[2] = {0.0, 0.0};
-#pragma unroll
-        for (int kk = 0; kk < W2 / 4; ++kk)
-          dmma884(acc, ss.S[(8 * i + (lane >> 2)) * BS + 4 * kk + (lane & 3)],
-                  ss.B[(4 * kk + (lane & 3)) * BS + 8 * j + (lane >> 2)]);
-#pragma unroll
-        for (int e = 0; e < 2; ++e)
-          jn[ii][j][e] = fma(-0.5, acc[e], ss.S[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e]);
-      }
-    named_bar(bar_id, 64);  // S is consumed by both warps: the fragments may overwrite it
-    // J'[r][c] -> fragment (kk = r / 4, nb = c / 8) slot of lane 4 (c % 8) + r % 4
-#pragma unroll
-    for (int ii = 0; ii < 2; ++ii)
-#pragma unroll
-      for (int j = 0; j < CG; ++j)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int r = 8 * (2 * HC + ii) + (lane >> 2), c = 8 * j + 2 * (lane & 3) + e;
-          ss.jf[((r >> 2) * CG + j) * 32 + 4 * (c & 7) + (r & 3)] = jn[ii][j][e];
-        }
-  }
-  named_bar(bar_id, 64);
-  PHASE_MARK(3);
-  // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J over this warp's rows.
-  apply_split(ss.ring, Wm + r0, ld, nr, I, J, lane, ss.jf);
-  PHASE_MARK(4);
-  const int hv = split_rows(vrows);
-  apply_split(ss.ring, Vm + (HC ? hv : 0), ldv, HC ? vrows - hv : hv, I, J, lane, ss.jf);
-  PHASE_MARK(5);
-  return true;
+// Per-warp shared-memory stride: the pair buffers, or a 32 x 33 transpose tile for the stage-in.
+template <int W2>
+__host__ __device__ constexpr size_t warp_stride() {
+  return ((WarpSmem<W2>::bytes() > 32 * 33 * 8 ? WarpSmem<W2>::bytes() : 32 * 33 * 8) + 15) & ~size_t(15);
 }
 
 }  // namespace
 
-template <int W2, int NW, typename TI, int GW>
-__global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
-                                                             const int* __restrict__ order) {
+// MODE: kFlat (flat Gram path, one CTA per matrix), kFlatCluster (flat Gram path, a cluster of CTAs
+// per matrix), kWcycle (Level 1 -> Level 2 recursion, one CTA). Separate instantiations keep one
+// inlined copy of process_pair per kernel (register pressure).
+enum { kFlat = 0, kFlatCluster = 1, kWcycle = 2 };
+
+template <int W2, int NW, typename TI, int MODE>
+__global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
+                                                             const int* __restrict__ order, SlotPool pool) {
   // TI: type of A, S, U, V in the caller's memory (double, or float for wcsvd_batched_f32); the
-  // iteration always runs on the fp64 working copy. GW: warps per column-block pair (1, or 2 =
-  // split executor, flat Gram path with 2w = 32 only).
-  static_assert(GW == 1 || (GW == 2 && W2 == kSplitW2 && NW % 2 == 0), "split executor: 2w = 32");
+  // iteration always runs on the fp64 working copy. CLU: the matrix is owned by a CTA cluster.
+  constexpr bool CLU = MODE == kFlatCluster;
   using C = PairCfg<W2>;
-  const MatDesc d = descs[order[blockIdx.x]];
+  const unsigned crank = CLU ? cl_rank() : 0u;
+  const int CL = CLU ? (int)cl_nrank() : 1;
+  const int mat = CLU ? (int)cl_id() : (int)blockIdx.x;
+  const MatDesc d = descs[order[mat]];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   constexpr int T = NW * 32;
+  const int gw = (int)crank * NW + warp;  // warp id inside the matrix's cluster
+  const int NWT = CL * NW;                // warps working on the matrix
   const int M = d.M, N = d.N, mp = d.m_pad, np = d.n_pad;
-  double* Wm = d.W;
-  double* Vm = d.Vw;
 
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WarpSmem<W2> ws;
-  SplitSmem ss;
-  if constexpr (GW == 2) {
-    unsigned char* p = smem_raw + (warp >> 1) * SplitSmem::bytes();
-    ss.B = reinterpret_cast<double*>(p);
-    ss.S = ss.B + 2 * W2 * W2;
-    ss.jf = ss.S;
-    ss.ring = ss.B + (warp & 1) * kSplitNS * kSplitSlab;
-    ss.red = ss.B + kSplitNS * kSplitSlab;
-    ss.cs = reinterpret_cast<double2*>(p + SplitSmem::region()) + (warp & 1) * (W2 / 2);
-    ss.xch = reinterpret_cast<double*>(reinterpret_cast<double2*>(p + SplitSmem::region()) + W2);
-  } else {
-    unsigned char* p = smem_raw + warp * WarpSmem<W2>::bytes();
+  {
+    unsigned char* p = smem_raw + warp * warp_stride<W2>();
     ws.B = reinterpret_cast<double*>(p);
     ws.S = ws.B + W2 * C::BS;
     ws.ring = ws.B;
@@ -1007,117 +648,165 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
     ws.tt = reinterpret_cast<double*>(ws.cs + W2 / 2);
     ws.pq = reinterpret_cast<int2*>(ws.tt + W2 / 2);
   }
-  __shared__ int s_flags[4];
-  __shared__ int s_inner[NW];
-  __shared__ int s_grp[2 * NW];
+  // Matrix-wide state (rank 0's copy is the one in use when CLU).
+  __shared__ int s_flags[4];          // [0, 1] sweep votes (parity), [2] non-finite, [3] needs completion
+  __shared__ int s_inner;             // total inner sweeps
+  __shared__ int s_slot;              // workspace slot of the matrix
+  __shared__ int s_grp[2 * NW];       // W-cycle group votes
   __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
-  __shared__ EvdMap<W2> s_em[32];     // inner-EVD work map per lane
+  __shared__ unsigned long long s_max;
+  __shared__ EvdMap<W2> s_em[32];     // inner-EVD work map per lane (per CTA)
   if (tid < 32) s_em[tid].init(tid);
   if (tid < 4) s_flags[tid] = 0;
-  if (tid < NW) s_inner[tid] = 0;
   if (tid < 2 * NW) s_grp[tid] = 0;
+  const int nb = np / C::W;
+  for (int b = tid; b < nb; b += T) s_blkver[b] = 0;
+  if (tid == 0) {
+    s_inner = 0;
+    s_max = 0ull;
+    if (crank == 0) s_slot = slot_acquire(pool, mat);
+  }
+  int* flags0 = s_flags;
+  int* ver0 = s_blkver;
+  int* inner0 = &s_inner;
+  unsigned long long* max0 = &s_max;
+  if constexpr (CLU) {
+    flags0 = at_rank0(s_flags);
+    ver0 = at_rank0(s_blkver);
+    inner0 = at_rank0(&s_inner);
+    max0 = at_rank0(&s_max);
+    cl_sync();
+  } else {
+    __syncthreads();
+  }
+  const int slot = CLU ? *at_rank0(&s_slot) : s_slot;
+  double* Wm = pool.base + (size_t)slot * pool.slot_doubles;
+  double* Vm = Wm + (size_t)mp * np;
 
-  // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. ----
-  __shared__ unsigned long long s_max;
-  if (tid == 0) s_max = 0ull;
-  __syncthreads();
+  // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. 32 x 32 tiles
+  // per warp; the transpose (m < n) goes through a shared-memory tile so that both the reads of A
+  // and the writes of W are coalesced. ----
   bool bad = false;
   double amax = 0.0;
-  for (size_t e = tid; e < (size_t)mp * np; e += T) {
-    const int c = (int)(e / mp), r = (int)(e % mp);
-    double v = 0.0;
-    if (r < M && c < N) {
-      const TI* Ain = reinterpret_cast<const TI*>(d.A);
-      v = (double)(d.swapped ? Ain[(size_t)r * d.lda + c] : Ain[(size_t)c * d.lda + r]);
-      bad |= !isfinite(v);
-      amax = fmax(amax, fabs(v));
+#ifdef WCSVD_EXP_STAGE_OLD
+  if (!CLU) {
+    for (size_t e = tid; e < (size_t)mp * np; e += T) {
+      const int c = (int)(e / mp), r = (int)(e % mp);
+      double v = 0.0;
+      if (r < M && c < N) {
+        const TI* Ain = reinterpret_cast<const TI*>(d.A);
+        v = (double)(d.swapped ? Ain[(size_t)r * d.lda + c] : Ain[(size_t)c * d.lda + r]);
+        bad |= !isfinite(v);
+        amax = fmax(amax, fabs(v));
+      }
+      Wm[e] = v;
     }
-    Wm[e] = v;
+  } else
+#endif
+  {
+    const TI* Ain = reinterpret_cast<const TI*>(d.A);
+    double* tile = reinterpret_cast<double*>(smem_raw + warp * warp_stride<W2>());
+    const int ntr = (mp + 31) / 32, ntc = (np + 31) / 32;
+    for (int t = gw; t < ntr * ntc; t += NWT) {
+      const int r0 = (t % ntr) * 32, c0 = (t / ntr) * 32;
+      if (d.swapped) {
+        // W row r = A column r; lane -> A row c0 + lane (contiguous)
+        for (int rr = 0; rr < 32; ++rr) {
+          const int r = r0 + rr, c = c0 + lane;
+          double v = 0.0;
+          if (r < M && c < N) {
+            v = (double)Ain[(size_t)r * d.lda + c];
+            bad |= !isfinite(v);
+            amax = fmax(amax, fabs(v));
+          }
+          tile[rr * 33 + lane] = v;
+        }
+        __syncwarp();
+        for (int cc = 0; cc < 32; ++cc) {
+          const int c = c0 + cc, r = r0 + lane;
+          if (r < mp && c < np) Wm[(size_t)c * mp + r] = tile[lane * 33 + cc];
+        }
+        __syncwarp();
+      } else {
+        for (int cc = 0; cc < 32; ++cc) {
+          const int c = c0 + cc, r = r0 + lane;
+          if (r < mp && c < np) {
+            double v = 0.0;
+            if (r < M && c < N) {
+              v = (double)Ain[(size_t)c * d.lda + r];
+              bad |= !isfinite(v);
+              amax = fmax(amax, fabs(v));
+            }
+            Wm[(size_t)c * mp + r] = v;
+          }
+        }
+      }
+    }
   }
   if (d.withv)
-    for (size_t e = tid; e < (size_t)np * np; e += T) Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
+    for (size_t e = (size_t)crank * T + tid; e < (size_t)np * np; e += (size_t)CL * T)
+      Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
   const int vrows = d.withv ? np : 0;  // values / U-only mode: V_x is not accumulated (§8(f4))
-  if (bad) atomicOr(&s_flags[2], 1);
-  if (amax > 0.0) atomicMax(&s_max, (unsigned long long)__double_as_longlong(amax));
-  __syncthreads();
-  const bool nonfinite = s_flags[2] != 0;
-  // Exact power-of-two pre-scaling to max|w| in [0.5, 1) (see l0_jacobi.cu).
+  if (bad) atomicOr(&flags0[2], 1);
+  if (amax > 0.0) atomicMax(max0, (unsigned long long)__double_as_longlong(amax));
+  if constexpr (CLU) cl_sync(); else __syncthreads();
+  const bool nonfinite = (CLU ? *(volatile int*)&flags0[2] : s_flags[2]) != 0;
+  const unsigned long long gmax = CLU ? *(volatile unsigned long long*)max0 : s_max;
+  // Exact power-of-two pre-scaling to max|w| in [0.5, 1) (see l0_jacobi.cu); every
+  // warp scales the tiles it wrote.
   int sexp = 0;
-  if (!nonfinite && s_max != 0ull) {
-    frexp(__longlong_as_double((long long)s_max), &sexp);
+  if (!nonfinite && gmax != 0ull) {
+    frexp(__longlong_as_double((long long)gmax), &sexp);
     const double f = ldexp(1.0, -sexp);
-    for (size_t e = tid; e < (size_t)mp * np; e += T) Wm[e] *= f;
+    const int ntr = (mp + 31) / 32, ntc = (np + 31) / 32;
+    for (int t = gw; t < ntr * ntc; t += NWT) {
+      const int r0 = (t % ntr) * 32, c0 = (t / ntr) * 32, r = r0 + lane;
+      if (r < mp)
+        for (int cc = 0; cc < 32 && c0 + cc < np; ++cc) Wm[(size_t)(c0 + cc) * mp + r] *= f;
+    }
   }
-  __syncthreads();
+  if constexpr (CLU) cl_sync(); else __syncthreads();
   const double tol2 = d.tol * d.tol;
-
 
   int sweep = 0;
   bool converged = false;
   int my_inner = 0;
-  if (!nonfinite && d.w2 == 0) {
+  if (MODE != kWcycle && !nonfinite) {
     // Flat Level 1: round-robin over the n_pad / w column blocks (Alg 1). Pairs are
-    // scheduled by dataflow instead of a CTA barrier per step: blk_ver[b] counts the pairs block b
-    // has completed, and the pair (I, J) of global step g starts once both blocks reached g. Each
-    // warp takes its pairs in (step, pair) order, so waits only point backwards (no deadlock), and
-    // warps drift into different phases (EVD overlaps other warps' DMMA work). The arithmetic of
-    // every pair is unchanged, so the result is bitwise that of the barrier schedule.
-    const int nb = np / C::W;
-    int* blk_ver = s_blkver;
-    for (int b = tid; b < nb; b += T) blk_ver[b] = 0;
-    __syncthreads();
+    // scheduled by dataflow instead of a barrier per step: ver[b] counts the pairs block b has
+    // completed, and the pair (I, J) of global step g starts once both blocks reached g. Each warp
+    // takes its pairs in (step, pair) order, so waits only point backwards (no deadlock), and warps
+    // drift into different phases (EVD overlaps other warps' DMMA work). The arithmetic of every pair
+    // is unchanged, so the result is bitwise that of a barrier schedule on any number of CTAs.
     int gstep = 0;
     while (sweep < d.max_sweeps) {
       bool rot_any = false;
       for (int step = 0; step < nb - 1; ++step, ++gstep) {
-        if constexpr (GW == 2) {
-          // split executor: group g = warp / 2 owns pairs g, g + NW/2, ...; warp 0 of the group
-          // acquires / releases, the group's named barrier orders both warps around the pair.
-          const int grp = warp >> 1, hc = warp & 1, bar = 1 + grp;
-          for (int p = grp; p < nb / 2; p += NW / 2) {
-            const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
-            if (hc == 0 && lane == 0) {
-              while (atomicAdd(&blk_ver[I], 0) < gstep || atomicAdd(&blk_ver[J], 0) < gstep) __nanosleep(20);
-            }
-            named_bar(bar, 64);
-            __threadfence_block();
-            rot_any |= hc ? process_pair_split<1>(ss, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, bar, &my_inner)
-                          : process_pair_split<0>(ss, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, bar, &my_inner);
-            __syncwarp();
-            __threadfence_block();
-            named_bar(bar, 64);
-            if (hc == 0 && lane == 0) {
-              atomicExch(&blk_ver[I], gstep + 1);
-              atomicExch(&blk_ver[J], gstep + 1);
-            }
-          }
-        } else {
-        for (int p = warp; p < nb / 2; p += NW) {
+        for (int p = gw; p < nb / 2; p += NWT) {
           const int I = rr_content(2 * p, step, nb), J = rr_content(2 * p + 1, step, nb);
-          if (lane == 0) {  // acquire: relaxed atomic reads, then a fence
-            while (atomicAdd(&blk_ver[I], 0) < gstep || atomicAdd(&blk_ver[J], 0) < gstep) __nanosleep(20);
+          if (lane == 0) {  // acquire
+            while (ver_acquire<CLU>(&ver0[I]) < gstep || ver_acquire<CLU>(&ver0[J]) < gstep) __nanosleep(20);
           }
           __syncwarp();
-          __threadfence_block();  // the previous owners' W / V writes are visible to every lane
+          pair_fence<CLU>();  // the previous owners' W / V writes are visible to every lane
           rot_any |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
-          __syncwarp();           // every lane's W / V writes precede ...
-          __threadfence_block();  // ... this fence, then the release (relaxed atomic store)
-          if (lane == 0) {
-            atomicExch(&blk_ver[I], gstep + 1);
-            atomicExch(&blk_ver[J], gstep + 1);
+          pair_fence<CLU>();  // every lane's W / V writes precede ...
+          __syncwarp();
+          if (lane == 0) {    // ... the release
+            ver_release<CLU>(&ver0[I], gstep + 1);
+            ver_release<CLU>(&ver0[J], gstep + 1);
           }
-        }
         }
       }
       ++sweep;
-      if (rot_any && lane == 0) s_flags[sweep & 1] = 1;
-      __syncthreads();
-      const bool any = s_flags[sweep & 1] != 0;
-      __syncthreads();
-      if (tid == 0) s_flags[sweep & 1] = 0;
+      if (rot_any && lane == 0) atomicOr(&flags0[sweep & 1], 1);
+      if constexpr (CLU) cl_sync(); else __syncthreads();
+      const bool any = (CLU ? *(volatile int*)&flags0[sweep & 1] : s_flags[sweep & 1]) != 0;
+      if constexpr (CLU) cl_sync(); else __syncthreads();
+      if (crank == 0 && tid == 0) s_flags[sweep & 1] = 0;
       if (!any) { converged = true; break; }
     }
-  } else if (GW == 1 && !nonfinite) {
+  } else if (MODE == kWcycle && !nonfinite) {
     // W-cycle (Alg 2 l.12-14; Step 3; Fig 3-4): Level-1 super-blocks
     // of width w1 = d.w are paired round-robin; each super-pair panel [A_I A_J] (M x 2 w1) fits no
     // on-chip EVD, so it recurses to Level 2: block Jacobi with w2 = d.w2 (the EVD width W2/2) over
@@ -1128,7 +817,7 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
     const int r = d.w / C::W;
     const int nb1 = np / d.w;
     const int GS = (r < NW) ? r : NW, NG = NW / GS;
-    const int grp = warp / GS, gw = warp % GS;
+    const int grp = warp / GS, gwi = warp % GS;
     const bool active_grp = grp < NG;
     while (sweep < d.max_sweeps) {
       bool rot_any = false;
@@ -1139,7 +828,7 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
             for (int isw = 0; isw < d.inner_cap2; ++isw) {
               bool mine = false;
               for (int s2 = 0; s2 < 2 * r - 1; ++s2) {
-                for (int p2 = gw; p2 < r; p2 += GS) {
+                for (int p2 = gwi; p2 < r; p2 += GS) {
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
@@ -1152,7 +841,7 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
               named_bar(1 + grp, GS * 32);
               const bool any2 = s_grp[grp * 2 + (isw & 1)] != 0;
               named_bar(1 + grp, GS * 32);
-              if (gw == 0 && lane == 0) s_grp[grp * 2 + (isw & 1)] = 0;
+              if (gwi == 0 && lane == 0) s_grp[grp * 2 + (isw & 1)] = 0;
               rot_any |= any2;
               if (!any2) break;
             }
@@ -1169,17 +858,28 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
       if (!any) { converged = true; break; }
     }
   }
-  if (lane == 0) s_inner[warp] = my_inner;
-  __syncthreads();
+  if (lane == 0 && my_inner) atomicAdd(inner0, my_inner);
 
   // ---- Finalisation: sigma, rank, sign (Z15), U = W / sigma, un-orientation. ----
+  // sigma and the sign of every column go to rank 0's arrays; every CTA then copies them locally.
   double* s_sig = reinterpret_cast<double*>(smem_raw);  // reuse warp buffers: [N]
   double* s_sgn = s_sig + N;                             // [N]
-  int* s_rank = reinterpret_cast<int*>(s_sgn + N);       // [N]
-  for (int j = warp; j < N; j += NW) {
+  double* sig0 = s_sig;
+  double* sgn0 = s_sgn;
+  if constexpr (CLU) {
+    cl_sync();  // every CTA is done with its warp buffers before rank 0's are overwritten
+    sig0 = at_rank0(s_sig);
+    sgn0 = at_rank0(s_sgn);
+  } else {
+    __syncthreads();
+  }
+  for (int j = gw; j < N; j += NWT) {
     const double* col = Wm + (size_t)j * mp;
     double a = 0.0;
-    for (int r = lane; r < M; r += 32) a = fma(col[r], col[r], a);
+    for (int r = lane; r < M; r += 32) {
+      const double x = __ldcg(col + r);
+      a = fma(x, x, a);
+    }
     for (int off = 16; off > 0; off >>= 1) a += __shfl_xor_sync(0xffffffffu, a, off);
     // Z15 sign rule on the square factor V_x; without V (values / U-only mode) on the columns of X.
     const double* vc = d.withv ? Vm + (size_t)j * np : col;
@@ -1187,7 +887,7 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
     double best = 0.0;
     int bi = 0x7fffffff;
     for (int i = lane; i < vlen; i += 32) {
-      const double v = vc[i];
+      const double v = __ldcg(vc + i);
       if (fabs(v) > fabs(best)) { best = v; bi = i; }
     }
     for (int off = 16; off > 0; off >>= 1) {
@@ -1196,23 +896,17 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
       if (fabs(ob) > fabs(best) || (fabs(ob) == fabs(best) && oi < bi)) { best = ob; bi = oi; }
     }
     if (lane == 0) {
-      s_sig[j] = nonfinite ? __longlong_as_double(0x7ff8000000000000ULL) : sqrt(a);
-      s_sgn[j] = (best < 0.0) ? -1.0 : 1.0;
+      sig0[j] = nonfinite ? __longlong_as_double(0x7ff8000000000000ULL) : sqrt(a);
+      sgn0[j] = (best < 0.0) ? -1.0 : 1.0;
     }
   }
-  __syncthreads();
-  for (int j = tid; j < N; j += T) {
-    int rk = 0;
-    if (nonfinite) {
-      rk = j;
-    } else {
-      const double sj = s_sig[j];
-      for (int i = 0; i < N; ++i) {
-        const double si = s_sig[i];
-        rk += (si > sj) || (si == sj && i < j);
+  if constexpr (CLU) {
+    cl_sync();
+    if (crank != 0)
+      for (int j = tid; j < N; j += T) {
+        s_sig[j] = sig0[j];
+        s_sgn[j] = sgn0[j];
       }
-    }
-    s_rank[j] = rk;
   }
   __syncthreads();
   double sig1 = 0.0;
@@ -1224,60 +918,93 @@ __global__ void __launch_bounds__(NW * 32, (GW == 2 && NW < 16) ? 16 / NW : 1) l
   TI* dstV = reinterpret_cast<TI*>(d.swapped ? d.U : d.V);
   const int ldV = d.swapped ? d.ldu : d.ldv;
   bool needs_completion = false;
-  for (int j = warp; j < N; j += NW) {
-    const int rk = s_rank[j];
+  for (int j = gw; j < N; j += NWT) {
+    // rank of column j in the stable descending order (ties to the lower index)
     const double sj = s_sig[j], sgn = s_sgn[j];
+    int rk = 0;
+    if (nonfinite) {
+      rk = j;
+    } else {
+      for (int i = lane; i < N; i += 32) {
+        const double si = s_sig[i];
+        rk += (si > sj) || (si == sj && i < j);
+      }
+      for (int off = 16; off > 0; off >>= 1) rk += __shfl_xor_sync(0xffffffffu, rk, off);
+    }
     const bool ok = sj > thresh;
     needs_completion |= !ok;
     if (dstW) {
       const double* col = Wm + (size_t)j * mp;
       for (int r = lane; r < M; r += 32)
-        dstW[(size_t)rk * ldW + r] = (TI)(nonfinite ? nanv : (ok ? sgn * (col[r] / sj) : sgn * 0.0));
+        dstW[(size_t)rk * ldW + r] = (TI)(nonfinite ? nanv : (ok ? sgn * (__ldcg(col + r) / sj) : sgn * 0.0));
     }
     if (dstV) {
       const double* vc = Vm + (size_t)j * np;
-      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = (TI)(nonfinite ? nanv : sgn * vc[i]);
+      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = (TI)(nonfinite ? nanv : sgn * __ldcg(vc + i));
     }
     if (lane == 0) reinterpret_cast<TI*>(d.S)[rk] = (TI)(nonfinite ? sj : ldexp(sj, sexp));
   }
-  if (needs_completion && !nonfinite && lane == 0) atomicOr(&s_flags[3], 1);
-  __syncthreads();
-  if (tid == 0) {
-    int inner = 0;
-    for (int w = 0; w < NW; ++w) inner += s_inner[w];
+  if (needs_completion && !nonfinite && lane == 0) atomicOr(&flags0[3], 1);
+  if constexpr (CLU) cl_sync(); else __syncthreads();
+  if (crank == 0 && tid == 0) {
     if (d.info) d.info[d.idx] = nonfinite ? -2 : (converged ? sweep : -1);
-    if (d.sweeps_inner) d.sweeps_inner[d.idx] = inner;
+    if (d.sweeps_inner) d.sweeps_inner[d.idx] = s_inner;
     if (d.status) d.status[d.idx] = (s_flags[3] && dstW) ? kNeedsCompletion : 0;
+    slot_release(pool, s_slot);
   }
 }
 
-template <int W2, int NW, typename TI, int GW>
-static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
-  size_t smem = (GW == 2) ? (NW / 2) * SplitSmem::bytes() : NW * WarpSmem<W2>::bytes();
-  const size_t fin = 3 * 8 * 1024;  // finalisation arrays alias the warp buffers
+template <int W2, int NW, typename TI, int MODE>
+static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, int cluster, const SlotPool& pool,
+                               cudaStream_t stream) {
+  size_t smem = NW * warp_stride<W2>();
+  const size_t fin = 2 * 8 * 1024;  // finalisation arrays alias the warp buffers
   if (smem < fin) smem = fin;
-  auto kern = l1_gram_kernel<W2, NW, TI, GW>;
+  auto kern = l1_gram_kernel<W2, NW, TI, MODE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  kern<<<count, NW * 32, smem, stream>>>(descs, order);
-  return cudaGetLastError();
+  if (MODE != kFlatCluster) {
+    kern<<<count, NW * 32, smem, stream>>>(descs, order, pool);
+    return cudaGetLastError();
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(count * cluster), 1, 1);
+  cfg.blockDim = dim3(NW * 32, 1, 1);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)cluster;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, descs, order, pool);
+}
+
+template <typename TI, int W2, int NW>
+static cudaError_t launch_l1_m(int wcycle, const MatDesc* descs, const int* order, int count, int cluster,
+                               const SlotPool& pool, cudaStream_t stream) {
+  if (wcycle) return launch_l1_t<W2, NW, TI, kWcycle>(descs, order, count, 1, pool, stream);
+  if (cluster > 1) return launch_l1_t<W2, NW, TI, kFlatCluster>(descs, order, count, cluster, pool, stream);
+  return launch_l1_t<W2, NW, TI, kFlat>(descs, order, count, 1, pool, stream);
 }
 
 template <typename TI>
-static cudaError_t launch_l1_v(int variant, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
+static cudaError_t launch_l1_v(int variant, int wcycle, const MatDesc* descs, const int* order, int count,
+                               int cluster, const SlotPool& pool, cudaStream_t stream) {
   switch (variant) {
-    case kL1_16x4: return launch_l1_t<16, 4, TI, 1>(descs, order, count, stream);
-    case kL1_32x4: return launch_l1_t<32, 4, TI, 1>(descs, order, count, stream);
-    case kL1_32x8: return launch_l1_t<32, 8, TI, 1>(descs, order, count, stream);
-    case kL1S_32x8: return launch_l1_t<32, 8, TI, 2>(descs, order, count, stream);
-    case kL1S_32x16: return launch_l1_t<32, 16, TI, 2>(descs, order, count, stream);
+    case kL1_16x4: return launch_l1_m<TI, 16, 4>(wcycle, descs, order, count, cluster, pool, stream);
+    case kL1_32x4: return launch_l1_m<TI, 32, 4>(wcycle, descs, order, count, cluster, pool, stream);
+    case kL1_32x8: return launch_l1_m<TI, 32, 8>(wcycle, descs, order, count, cluster, pool, stream);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_l1(int variant, int fp32, const MatDesc* descs, const int* order, int count, cudaStream_t stream) {
-  return fp32 ? launch_l1_v<float>(variant, descs, order, count, stream)
-              : launch_l1_v<double>(variant, descs, order, count, stream);
+cudaError_t launch_l1(int variant, int wcycle, int fp32, const MatDesc* descs, const int* order, int count,
+                      int cluster, const SlotPool& pool, cudaStream_t stream) {
+  return fp32 ? launch_l1_v<float>(variant, wcycle, descs, order, count, cluster, pool, stream)
+              : launch_l1_v<double>(variant, wcycle, descs, order, count, cluster, pool, stream);
 }
 
 }  // namespace wcsvd

@@ -58,8 +58,11 @@ def svd_batched_dist(sizes: Sequence, make_matrix: Callable[[int], "object"], ra
 
 def gather_sigma(indices: list, S: list, sizes: Sequence, group=None, dst: int = 0):
     """Gather every rank's singular values to rank `dst` (one collective, after the batch).
-    Returns the full list S[k] (k = 0..batch-1) on `dst`, None elsewhere. Works with any backend
-    (tensors are staged on the backend's device: CUDA for NCCL, CPU for gloo)."""
+    Returns the full list S[k] (k = 0..batch-1, CPU float64 tensors) on `dst`, None elsewhere.
+    Works with any backend: the padded [rows, 1 + kmax] block (column 0 = batch index) is packed on
+    the host, moved once to the backend's device (CUDA for NCCL, CPU for gloo) and gathered with one
+    all_gather (plus one tiny all_gather of the row counts)."""
+    import numpy as np
     import torch
     import torch.distributed as dist
 
@@ -68,22 +71,25 @@ def gather_sigma(indices: list, S: list, sizes: Sequence, group=None, dst: int =
     backend = dist.get_backend(group)
     dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
     kmax = max((min(m, n) for (m, n) in sizes), default=0)
-    nloc = torch.tensor([len(indices)], device=dev)
-    counts = [torch.zeros(1, dtype=nloc.dtype, device=dev) for _ in range(world)]
+    nloc = torch.tensor([len(indices)], dtype=torch.int64, device=dev)
+    counts = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(world)]
     dist.all_gather(counts, nloc, group=group)
-    cmax = int(max(c.item() for c in counts))
-    buf = torch.full((max(cmax, 1), kmax + 1), float("nan"), dtype=torch.float64, device=dev)
+    counts = [int(c.item()) for c in counts]
+    cmax = max(max(counts), 1)
+    host = np.full((cmax, kmax + 1), np.nan)
     for j, (k, s) in enumerate(zip(indices, S)):
-        buf[j, 0] = float(k)
-        buf[j, 1:1 + s.numel()] = s.to(dev)
+        host[j, 0] = float(k)
+        sv = s.detach().cpu().numpy() if isinstance(s, torch.Tensor) else np.asarray(s)
+        host[j, 1:1 + sv.size] = sv.reshape(-1)
+    buf = torch.from_numpy(host).to(dev)
     outs = [torch.empty_like(buf) for _ in range(world)]
     dist.all_gather(outs, buf, group=group)
     if rank != dst:
         return None
     full = [None] * len(sizes)
     for r in range(world):
-        for j in range(int(counts[r].item())):
-            k = int(outs[r][j, 0].item())
-            kk = min(sizes[k])
-            full[k] = outs[r][j, 1:1 + kk].cpu()
+        o = outs[r].cpu()
+        for j in range(counts[r]):
+            k = int(o[j, 0].item())
+            full[k] = o[j, 1:1 + min(sizes[k])].clone()
     return full

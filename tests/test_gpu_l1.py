@@ -111,18 +111,11 @@ def test_c5_mixed_sampled_and_1024_properties():
         assert np.abs(S[k] - s_ref).max() / s_ref[0] <= 1e-12
 
 
-def test_split_executor_pair_warps_2():
-    # Ablation path (wcsvd_opts.pair_warps = 2): two warps per column-block pair
-    # (row-split Gram / update, column halves of J, 64-lane EVD). Same oracle bars; deterministic.
-    shapes = [(256, 256), (300, 170), (170, 300), (1024, 128), (130, 99), (513, 257), (200, 120)]
-    mats = [workloads.gaussian(workloads.matrix_rng(570 + i, 2), m, n) for i, (m, n) in enumerate(shapes)]
-    S, U, V, info = gpu_svd_list(mats, pair_warps=2)
-    check_parity(mats, S, U, V, info)
-    S2, U2, V2, _ = gpu_svd_list(mats[::-1], pair_warps=2)
-    assert all(np.array_equal(S[i], S2[-1 - i]) and np.array_equal(U[i], U2[-1 - i]) for i in range(len(mats)))
-    # values-only mode on the split executor (V not accumulated)
+def test_removed_split_executor_is_rejected():
+    # wcsvd_opts.pair_warps = 2 (round-1 ablation executor) was removed: -12 before anything is enqueued
     import torch
     import paper_conf_sc_xiaopxsmmlzt22_b200 as wcm
-    A = torch.from_numpy(np.ascontiguousarray(mats[0])).cuda()[None]
-    Sv, _, _ = wcm.svd_batched(A, compute_uv=False, pair_warps=2)
-    assert np.array_equal(Sv.cpu().numpy()[0], S[0])
+    A = torch.from_numpy(workloads.gaussian(workloads.matrix_rng(570, 2), 256, 256)).cuda()[None]
+    with pytest.raises(wcm.WcsvdError) as ei:
+        wcm.svd_batched(A, pair_warps=2)
+    assert ei.value.code == -12

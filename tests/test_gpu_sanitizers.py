@@ -1,7 +1,7 @@
 """T8: compute-sanitizer memcheck / racecheck / synccheck / initcheck on a small mixed
 batch covering the Level-0 variants, the Level-1 Gram path (w = 8 and 16, dataflow pair scheduling,
-cp.async slab rings), the W-cycle path, the split pair executor (two warps sharing B, J halves and the
-Gram partials through shared memory) and the host-buffer pipeline."""
+cp.async slab rings), the W-cycle path, a Gram-path matrix spread over a 4-CTA cluster (dataflow
+counters and votes in distributed shared memory) and the host-buffer pipeline."""
 import os
 import shutil
 import subprocess
@@ -15,8 +15,8 @@ SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitize
 
 
 @pytest.mark.parametrize("tool,mode", [("memcheck", "mixed"), ("racecheck", "mixed"), ("racecheck", "wcycle"),
-                                       ("synccheck", "mixed"), ("initcheck", "mixed"), ("racecheck", "split"),
-                                       ("synccheck", "split"), ("synccheck", "wcycle"), ("memcheck", "host")])
+                                       ("synccheck", "mixed"), ("initcheck", "mixed"), ("racecheck", "cluster"),
+                                       ("synccheck", "cluster"), ("synccheck", "wcycle"), ("memcheck", "host")])
 def test_sanitizer_clean(tool, mode):
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not available")
