@@ -155,6 +155,25 @@ WCSVD_API int wcsvd_batched_host(int batch, const int* m, const int* n, const do
  * visible). 0 for an invalid batch. */
 WCSVD_API size_t wcsvd_workspace_size(int batch, const int* m, const int* n);
 
+/* wcsvd_etkf_analysis -- the data-assimilation consumer of the SVD (§V.F:
+ * one SVD per grid point of an ocean model, batched; the paper's DA codes are ensemble Kalman filters,
+ * refs [36]-[38] PAPER.md:538-541). Reading R-DA: the ETKF ensemble-space analysis.
+ * Per grid point b, with the scaled observation-space ensemble perturbations Y_b (m x n: m obs,
+ * n members) = U diag(S) V^T as returned by wcsvd_batched, and the scaled innovation d_b (m):
+ *   wbar = (I_n + Y^T Y)^-1 Y^T d = V diag(s / (1 + s^2)) U^T d             (n)
+ *   T    = (I_n + Y^T Y)^-1/2     = I_n + V diag((1 + s^2)^-1/2 - 1) V^T      (n x n, symmetric)
+ * so that the analysis ensemble is X_a = xbar_b 1^T + X_b' (wbar 1^T + T) (unscaled: see DESIGN.md).
+ *  m, n        host [batch], 1..1024.                                                     (2, 3)
+ *  S, U, V     host [batch] of DEVICE pointers: S k = min(m,n); U m x k (ld m); V n x k (ld n),
+ *              column-major -- exactly wcsvd_batched's outputs for Y_b.                   (4-6)
+ *  d           host [batch] of DEVICE pointers to m doubles.                               (7)
+ *  wbar, T     host [batch] of DEVICE output pointers: n doubles; n x n column-major (ld n). (8, 9)
+ * Asynchronous on `stream`; negative codes (argument index / ENOTSUP / ENOMEM / ECUDA) synchronous,
+ * nothing enqueued on an argument error. Deterministic (fixed-order sums, FP64 DMMA tiles). */
+WCSVD_API int wcsvd_etkf_analysis(int batch, const int* m, const int* n, const double* const* S,
+                                  const double* const* U, const double* const* V, const double* const* d,
+                                  double* const* wbar, double* const* T, wcsvd_stream_t stream);
+
 /* Release the cached blocks of the library's workspace pool on the current device (after pending
  * calls complete). Returns WCSVD_OK or WCSVD_ECUDA. */
 WCSVD_API int wcsvd_trim_workspace(void);

@@ -17,7 +17,7 @@ from typing import Sequence
 
 import numpy as np
 
-__all__ = ["svd_batched", "svd_batched_host", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
+__all__ = ["svd_batched", "svd_batched_host", "etkf_analysis", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
            "PATH_L0", "PATH_GRAM", "PATH_WCYCLE", "L0_TWO_PHASE_VARIANTS", "library_path"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -84,6 +84,8 @@ def lib() -> ctypes.CDLL:
     L.wcsvd_round_robin.argtypes = [I, I, P]
     L.wcsvd_round_robin.restype = I
     L.wcsvd_version.restype = ctypes.c_char_p
+    L.wcsvd_etkf_analysis.argtypes = [I, P, P, P, P, P, P, P, P, P]
+    L.wcsvd_etkf_analysis.restype = I
     L.wcsvd_trim_workspace.argtypes = []
     L.wcsvd_trim_workspace.restype = I
     _lib = L
@@ -108,6 +110,17 @@ def round_robin(np_: int, step: int) -> list:
     if lib().wcsvd_round_robin(int(np_), int(step), buf) != 0:
         raise ValueError("bad round-robin arguments")
     return [(buf[2 * k], buf[2 * k + 1]) for k in range(np_ // 2)]
+
+
+def _check_out(t, shape, dtype, cuda: bool, name: str):
+    """A caller-supplied output buffer must match exactly (the C-ABI writes through raw pointers)."""
+    if t is None:
+        return
+    if tuple(t.shape) != tuple(shape) or t.dtype != dtype or not t.is_contiguous() or bool(t.is_cuda) != cuda:
+        where = "CUDA" if cuda else "host"
+        raise ValueError(f"out buffer {name}: expected a contiguous {where} {dtype} tensor of shape "
+                         f"{tuple(shape)}, got {tuple(t.shape)} {t.dtype} contiguous={t.is_contiguous()} "
+                         f"cuda={t.is_cuda}")
 
 
 def _arr_i32(x) -> np.ndarray:
@@ -185,6 +198,12 @@ def svd_batched(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool = Tru
         es = A.element_size()
         if out is not None:
             S, Ubuf, Vbuf = out
+            _check_out(S, (B, k), dt, True, "S")
+            _check_out(Ubuf, (B, k, m), dt, True, "U")
+            _check_out(Vbuf, (B, k, n), dt, True, "V")
+            for t in (S, Ubuf, Vbuf):
+                if t is not None and t.device != dev:
+                    raise ValueError("out buffers must be on the device of A")
         else:
             S = torch.empty(B, k, dtype=dt, device=dev)
             Ubuf = torch.empty(B, k, m, dtype=dt, device=dev) if cu else None
@@ -276,6 +295,9 @@ def svd_batched_host(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool 
         k = min(m, n)
         if out is not None:
             S, Ubuf, Vbuf = out
+            _check_out(S, (B, k), A.dtype, False, "S")
+            _check_out(Ubuf, (B, k, m), A.dtype, False, "U")
+            _check_out(Vbuf, (B, k, n), A.dtype, False, "V")
         else:
             pin = A.is_pinned()
             S = torch.empty(B, k, dtype=A.dtype, pin_memory=pin)
@@ -306,6 +328,12 @@ def svd_batched_host(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool 
     ks = [min(x, y) for x, y in zip(ms, ns)]
     if out is not None:  # lists (S, Ubuf, Vbuf) of host buffers [k], [k, m], [k, n]
         Ss, Ub, Vb = out
+        if len(Ss) != B or (Ub is not None and len(Ub) != B) or (Vb is not None and len(Vb) != B):
+            raise ValueError("out lists must have one buffer per matrix")
+        for i in range(B):
+            _check_out(Ss[i], (ks[i],), torch.float64, False, f"S[{i}]")
+            _check_out(Ub[i] if Ub is not None else None, (ks[i], ms[i]), torch.float64, False, f"U[{i}]")
+            _check_out(Vb[i] if Vb is not None else None, (ks[i], ns[i]), torch.float64, False, f"V[{i}]")
     else:
         Ss = [torch.empty(k, dtype=torch.float64, pin_memory=pin) for k in ks]
         Ub = [torch.empty(k, mm, dtype=torch.float64, pin_memory=pin) for k, mm in zip(ks, ms)] if compute_uv else None
@@ -317,3 +345,61 @@ def svd_batched_host(A, tol: float = 0.0, max_sweeps: int = 0, compute_uv: bool 
     Us = [u.T for u in Ub] if Ub is not None else None
     Vs = [v.T for v in Vb] if Vb is not None else None
     return (Ss, Us, Vs, info) if return_info else (Ss, Us, Vs)
+
+
+def etkf_analysis(S, U, V, d):
+    """Data-assimilation consumer (wcsvd_etkf_analysis): for each grid
+    point with scaled ensemble perturbations Y = U diag(S) V^T (svd_batched's outputs) and scaled
+    innovation d, returns (wbar, T) with wbar = (I + Y^T Y)^-1 Y^T d and T = (I + Y^T Y)^-1/2.
+
+    Batched form: S [B, k], U [B, m, k], V [B, n, k] exactly as svd_batched returns them (U, V are
+    transposed views of contiguous buffers), d [B, m] -> wbar [B, n], T [B, n, n]. List form: lists of
+    the per-matrix tensors -> lists. fp64 CUDA tensors; runs on the current stream."""
+    import torch
+
+    if not torch.cuda.is_available():
+        raise WcsvdError(WCSVD_ECUDA, "no CUDA device (this library has no CPU fallback)")
+    stream = torch.cuda.current_stream().cuda_stream
+    batched = isinstance(S, torch.Tensor)
+    Ss = list(S) if batched else list(S)
+    Us = list(U) if batched else list(U)
+    Vs = list(V) if batched else list(V)
+    ds = list(d) if batched else list(d)
+    B = len(Ss)
+    if not (len(Us) == len(Vs) == len(ds) == B):
+        raise ValueError("S, U, V, d must have one entry per matrix")
+    if B == 0:
+        return ([], []) if not batched else (None, None)
+    ms, ns, ptrs = [], [], {"S": [], "U": [], "V": [], "d": []}
+    keep = []
+    for s, u, v, dd in zip(Ss, Us, Vs, ds):
+        for t in (s, u, v, dd):
+            if t.dtype != torch.float64 or not t.is_cuda:
+                raise ValueError("S, U, V, d must be float64 CUDA tensors")
+        m, k = u.shape
+        n = v.shape[0]
+        if v.shape[1] != k or s.numel() != k or k != min(m, n) or dd.numel() != m:
+            raise ValueError("shapes must be S [k], U [m, k], V [n, k], d [m] with k = min(m, n)")
+        uc, vc = u.t().contiguous(), v.t().contiguous()  # column-major m x k / n x k (no copy for views)
+        sc, dc = s.contiguous(), dd.contiguous()
+        keep += [uc, vc, sc, dc]
+        ms.append(m)
+        ns.append(n)
+        ptrs["S"].append(sc.data_ptr())
+        ptrs["U"].append(uc.data_ptr())
+        ptrs["V"].append(vc.data_ptr())
+        ptrs["d"].append(dc.data_ptr())
+    dev = Ss[0].device
+    wb = [torch.empty(n, dtype=torch.float64, device=dev) for n in ns]
+    Tb = [torch.empty(n, n, dtype=torch.float64, device=dev) for n in ns]  # written column-major
+    mm, nn = _arr_i32(ms), _arr_i32(ns)
+    arr = {k: _arr_ptr(v) for k, v in ptrs.items()}
+    pw = _arr_ptr([w.data_ptr() for w in wb])
+    pt = _arr_ptr([t.data_ptr() for t in Tb])
+    _check(lib().wcsvd_etkf_analysis(B, mm.ctypes.data, nn.ctypes.data, arr["S"].ctypes.data, arr["U"].ctypes.data,
+                                     arr["V"].ctypes.data, arr["d"].ctypes.data, pw.ctypes.data, pt.ctypes.data,
+                                     stream or None))
+    Ts = [t.t() for t in Tb]
+    if batched:
+        return torch.stack(wb), torch.stack(Ts)
+    return wb, Ts

@@ -158,8 +158,10 @@ struct CallPlan {
   size_t off_descs = 0, off_order = 0, off_status = 0, bytes = 0;
 };
 
+// tot_cost > 0: the tailoring shares are taken against this total (the host pipeline plans each chunk
+// against the whole batch, whose chunks run concurrently), else against this call's own batch.
 int make_call_plan(int batch, const int* m, const int* n, int force_path, int force_w, int force_cluster,
-                   const std::vector<int>* withv, CallPlan* cp) {
+                   const std::vector<int>* withv, CallPlan* cp, double tot_cost = 0.0) {
   cp->plans.assign(batch, wcsvd_plan_t{});
   double tot = 0;
   for (int b = 0; b < batch; ++b) {
@@ -167,6 +169,7 @@ int make_call_plan(int batch, const int* m, const int* n, int force_path, int fo
     if (rc != WCSVD_OK) return rc;
     tot += cp->plans[b].cost;
   }
+  if (tot_cost > 0) tot = tot_cost;
   const int sms = device_sms();
   auto& buckets = cp->buckets;
   buckets.clear();
@@ -306,7 +309,7 @@ using namespace wcsvd;
 template <typename TI>
 static int batched_impl(int batch, const int* m, const int* n, const TI* const* A, const int* lda,
                         TI* const* S, TI* const* U, TI* const* V, double tol, int max_sweeps,
-                        wcsvd_stream_t stream_, const wcsvd_opts* opts) {
+                        wcsvd_stream_t stream_, const wcsvd_opts* opts, double tailor_total = 0.0) {
   constexpr bool kF32 = sizeof(TI) == 4;
   const double eps = kF32 ? 5.9604644775390625e-08 : kU53;  // 2^-24 or 2^-53
   cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
@@ -326,7 +329,8 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
   for (int b = 0; b < batch; ++b)
     withv[b] = (m[b] < n[b]) ? (U && U[b] ? 1 : 0) : (V && V[b] ? 1 : 0);
   CallPlan cp;
-  const int rc0 = make_call_plan(batch, m, n, force_path, force_w, opts ? opts->cluster_ctas : 0, &withv, &cp);
+  const int rc0 = make_call_plan(batch, m, n, force_path, force_w, opts ? opts->cluster_ctas : 0, &withv, &cp,
+                                 tailor_total);
   if (rc0 != WCSVD_OK) return rc0;
   const auto& plans = cp.plans;
   const auto& buckets = cp.buckets;
@@ -705,7 +709,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
     }
     rc = batched_impl<double>(cnt, m + b0, n + b0, pA.data(), ld_.data(), pS.data(), wantU ? pU.data() : nullptr,
                               wantV ? pV.data() : nullptr, tol, max_sweeps,
-                              reinterpret_cast<wcsvd_stream_t>(s_cp[cs]), &o);
+                              reinterpret_cast<wcsvd_stream_t>(s_cp[cs]), &o, tot);
     if (rc != WCSVD_OK) break;
     e = cudaEventRecord(ev_cp[st], s_cp[cs]);
     // D2H of the previous chunk now (a copy to pageable host memory returns only when it is done, so
@@ -798,6 +802,50 @@ size_t wcsvd_workspace_size(int batch, const int* m, const int* n) {
   CallPlan cp;
   if (make_call_plan(batch, m, n, 0, 0, 0, nullptr, &cp) != WCSVD_OK) return 0;
   return cp.bytes;
+}
+
+int wcsvd_etkf_analysis(int batch, const int* m, const int* n, const double* const* S, const double* const* U,
+                        const double* const* V, const double* const* d, double* const* wbar, double* const* T,
+                        wcsvd_stream_t stream_) {
+  cudaStream_t stream = reinterpret_cast<cudaStream_t>(stream_);
+  if (batch < 0) return -1;
+  if (batch == 0) return WCSVD_OK;
+  if (!m) return -2;
+  if (!n) return -3;
+  if (!S) return -4;
+  if (!U) return -5;
+  if (!V) return -6;
+  if (!d) return -7;
+  if (!wbar) return -8;
+  if (!T) return -9;
+  int kmax = 0;
+  std::vector<DaDesc> h(batch);
+  for (int b = 0; b < batch; ++b) {
+    if (m[b] < 1) return -2;
+    if (n[b] < 1) return -3;
+    if (!S[b]) return -4;
+    if (!U[b]) return -5;
+    if (!V[b]) return -6;
+    if (!d[b]) return -7;
+    if (!wbar[b]) return -8;
+    if (!T[b]) return -9;
+    if (m[b] > kMaxDim || n[b] > kMaxDim) return WCSVD_ENOTSUP;
+    h[b] = DaDesc{S[b], U[b], V[b], d[b], wbar[b], T[b], m[b], n[b]};
+    kmax = std::max(kmax, std::min(m[b], n[b]));
+  }
+  void* ws = nullptr;
+  if (lib_malloc(&ws, sizeof(DaDesc) * (size_t)batch, stream) != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ENOMEM;
+  }
+  cudaError_t e = cudaMemcpyAsync(ws, h.data(), sizeof(DaDesc) * (size_t)batch, cudaMemcpyHostToDevice, stream);
+  if (e == cudaSuccess) e = launch_etkf(static_cast<const DaDesc*>(ws), batch, kmax, stream);
+  cudaFreeAsync(ws, stream);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ECUDA;
+  }
+  return WCSVD_OK;
 }
 
 int wcsvd_trim_workspace(void) {

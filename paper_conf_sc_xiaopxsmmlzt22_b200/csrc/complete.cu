@@ -45,10 +45,14 @@ __global__ void __launch_bounds__(kCT) complete_u_kernel(const MatDesc* __restri
   __shared__ double red[kCT / 32];
   __shared__ double s_res[kCT / 32];
   __shared__ int s_idx[kCT / 32];
-  const double eps = sizeof(TI) == 4 ? 5.9604644775390625e-08 : kU53;
-  const double thresh = (double)S[0] * (double)M * eps;
+  (void)S;
   for (int k = 0; k < N; ++k) {
-    if ((double)S[k] > thresh) continue;
+    // Complete exactly the columns finalisation wrote as (signed) zeros: the finalising kernel applied
+    // its own rank threshold (sigma_1 M 2^-53 on the fp64 iterate, 2^-24 for the fp32 Level-0 kernel),
+    // so this pass never overwrites a valid column (a unit vector is never all zero).
+    int nz = 0;
+    for (int r = threadIdx.x; r < M; r += kCT) nz |= ((double)Uw[(size_t)k * ld + r] != 0.0);
+    if (__syncthreads_or(nz)) continue;
     const double sgn = signbit((double)Uw[(size_t)k * ld]) ? -1.0 : 1.0;  // Z15 flip recorded as -0.0
     // candidate e_i with the largest residual^2 = 1 - sum_{q<k} u_q[i]^2 (first i on ties)
     double bres = -1.0;

@@ -44,3 +44,17 @@ cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, co
 namespace wcsvd {
 cudaError_t launch_complete(int fp32, const MatDesc* descs, int count, cudaStream_t stream);
 }  // namespace wcsvd
+
+namespace wcsvd {
+// Data-assimilation consumer (da.cu): per grid point, the ETKF ensemble-space analysis from an SVD.
+struct DaDesc {
+  const double* S;  // k = min(m, n)
+  const double* U;  // m x k, ld m
+  const double* V;  // n x k, ld n
+  const double* d;  // m
+  double* wbar;     // n
+  double* T;        // n x n, ld n
+  int m, n;
+};
+cudaError_t launch_etkf(const DaDesc* descs, int count, int kmax, cudaStream_t stream);
+}  // namespace wcsvd

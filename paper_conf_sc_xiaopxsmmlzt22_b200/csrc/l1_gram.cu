@@ -585,8 +585,8 @@ __device__ __forceinline__ T* at_rank0(T* p) {
 template <bool CLU>
 __device__ __forceinline__ int ver_acquire(int* p) {
   if constexpr (CLU) {
-    int v;
-    asm volatile("ld.acquire.cluster.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    int v;  // an atomic read (atom.acquire, not ld.acquire): compute-sanitizer racecheck models atomics
+    asm volatile("atom.acquire.cluster.or.b32 %0, [%1], 0;" : "=r"(v) : "l"(p) : "memory");
     return v;
   } else {
     return atomicAdd(p, 0);  // relaxed read; the fence after the spin orders the panel reads
@@ -594,10 +594,12 @@ __device__ __forceinline__ int ver_acquire(int* p) {
 }
 template <bool CLU>
 __device__ __forceinline__ void ver_release(int* p, int v) {
-  if constexpr (CLU)
-    asm volatile("st.release.cluster.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-  else
+  if constexpr (CLU) {
+    int old;
+    asm volatile("atom.release.cluster.exch.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  } else {
     atomicExch(p, v);
+  }
 }
 template <bool CLU>
 __device__ __forceinline__ void pair_fence() {
@@ -655,6 +657,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __shared__ int s_grp[2 * NW];       // W-cycle group votes
   __shared__ int s_blkver[1024 / 8];  // per-block completed-pair counters (flat path)
   __shared__ unsigned long long s_max;
+  __shared__ unsigned long long s_clmax[8];  // rank 0: per-CTA max |a_ij| (bit 63 = non-finite seen)
   __shared__ EvdMap<W2> s_em[32];     // inner-EVD work map per lane (per CTA)
   if (tid < 32) s_em[tid].init(tid);
   if (tid < 4) s_flags[tid] = 0;
@@ -669,12 +672,10 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   int* flags0 = s_flags;
   int* ver0 = s_blkver;
   int* inner0 = &s_inner;
-  unsigned long long* max0 = &s_max;
   if constexpr (CLU) {
     flags0 = at_rank0(s_flags);
     ver0 = at_rank0(s_blkver);
     inner0 = at_rank0(&s_inner);
-    max0 = at_rank0(&s_max);
     cl_sync();
   } else {
     __syncthreads();
@@ -747,11 +748,21 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     for (size_t e = (size_t)crank * T + tid; e < (size_t)np * np; e += (size_t)CL * T)
       Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
   const int vrows = d.withv ? np : 0;  // values / U-only mode: V_x is not accumulated (§8(f4))
-  if (bad) atomicOr(&flags0[2], 1);
-  if (amax > 0.0) atomicMax(max0, (unsigned long long)__double_as_longlong(amax));
-  if constexpr (CLU) cl_sync(); else __syncthreads();
-  const bool nonfinite = (CLU ? *(volatile int*)&flags0[2] : s_flags[2]) != 0;
-  const unsigned long long gmax = CLU ? *(volatile unsigned long long*)max0 : s_max;
+  // max |a_ij| and the non-finite flag: CTA-local atomics, then (cluster) one slot per CTA in rank 0
+  if (bad) atomicOr(&s_flags[2], 1);
+  if (amax > 0.0) atomicMax(&s_max, (unsigned long long)__double_as_longlong(amax));
+  __syncthreads();
+  bool nonfinite = s_flags[2] != 0;
+  unsigned long long gmax = s_max;
+  if constexpr (CLU) {
+    if (tid == 0) at_rank0(s_clmax)[crank] = gmax | (nonfinite ? (1ull << 63) : 0ull);
+    cl_sync();
+    const unsigned long long* cm = at_rank0(s_clmax);
+    gmax = 0ull;
+    for (int r = 0; r < CL; ++r) gmax = (cm[r] & ~(1ull << 63)) > gmax ? (cm[r] & ~(1ull << 63)) : gmax;
+    nonfinite = false;
+    for (int r = 0; r < CL; ++r) nonfinite |= (cm[r] >> 63) != 0;
+  }
   // Exact power-of-two pre-scaling to max|w| in [0.5, 1) (see l0_jacobi.cu); every
   // warp scales the tiles it wrote.
   int sexp = 0;
@@ -862,12 +873,13 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
 
   // ---- Finalisation: sigma, rank, sign (Z15), U = W / sigma, un-orientation. ----
   // sigma and the sign of every column go to rank 0's arrays; every CTA then copies them locally.
-  double* s_sig = reinterpret_cast<double*>(smem_raw);  // reuse warp buffers: [N]
+  // one CTA: reuse the warp buffers; cluster: a dedicated region after them (other CTAs write rank 0's
+  // copy while its warps may still be draining their slab rings)
+  double* s_sig = reinterpret_cast<double*>(smem_raw + (CLU ? NW * warp_stride<W2>() : 0));  // [N]
   double* s_sgn = s_sig + N;                             // [N]
   double* sig0 = s_sig;
   double* sgn0 = s_sgn;
   if constexpr (CLU) {
-    cl_sync();  // every CTA is done with its warp buffers before rank 0's are overwritten
     sig0 = at_rank0(s_sig);
     sgn0 = at_rank0(s_sgn);
   } else {
@@ -958,8 +970,9 @@ template <int W2, int NW, typename TI, int MODE>
 static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, int cluster, const SlotPool& pool,
                                cudaStream_t stream) {
   size_t smem = NW * warp_stride<W2>();
-  const size_t fin = 2 * 8 * 1024;  // finalisation arrays alias the warp buffers
-  if (smem < fin) smem = fin;
+  const size_t fin = 2 * 8 * 1024;  // finalisation arrays: alias the warp buffers (one CTA) or follow them
+  if (MODE == kFlatCluster) smem += fin;
+  else if (smem < fin) smem = fin;
   auto kern = l1_gram_kernel<W2, NW, TI, MODE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
