@@ -108,6 +108,10 @@ typedef struct {
                               dominate the batch is spread over a thread-block cluster of 2, 4 or 8
                               CTAs); 1, 2, 4, 8 force the CTAs per Gram-path matrix (ablations).
                               Results are bitwise independent of it. Other values: -12 */
+  int f32_compute;         /* wcsvd_batched_f32 only: 0 = planner (Gram-path matrices iterate on an fp64
+                              working copy with FP64 DMMA contractions and are rounded at finalisation:
+                              the fastest on B200), 1 = iterate in fp32 (FFMA Gram / update, fp32 EVD and
+                              Newton-Schulz on an fp32 working copy; ablation). Other values: -12 */
 } wcsvd_opts;
 
 WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const double* const* A, const int* lda,
@@ -116,10 +120,13 @@ WCSVD_API int wcsvd_batched_ex(int batch, const int* m, const int* n, const doub
 
 /* wcsvd_batched_f32 / _f32_ex -- the fp32 variant: same arguments, layout,
  * ownership, errors and determinism as wcsvd_batched, with float data. tol <= 0 -> sqrt(max(m,n)) *
- * 2^-24. Level-0 matrices are iterated in fp32 throughout; Level-1 (Gram path) matrices are iterated
- * by the fp64 DMMA kernel on an fp64 working copy (sm_100a has no full-precision fp32 MMA) and
- * rounded to fp32 at finalisation. Accuracy targets (north_star): sigma 1e-5, residual 1e-5,
- * orthogonality 1e-4, all relative. */
+ * 2^-24. Level-0 matrices iterate in fp32 (FFMA). Gram-path matrices iterate, by default, on an fp64
+ * working copy with the FP64 DMMA contractions (sm_100a has no full-precision fp32 MMA: DMMA is
+ * fp64-only, TF32 keeps 10 mantissa bits; an FFMA contraction needs 8x the issue slots of DMMA per
+ * flop while the FP32 pipe is only 2x the FP64 one, so this is the fastest route) and are rounded to
+ * fp32 at finalisation; opts->f32_compute = 1 selects the all-fp32 Gram path (FFMA Gram / update, fp32
+ * EVD and Newton-Schulz on an fp32 working copy). Accuracy targets (north_star): sigma 1e-5, residual
+ * 1e-5, orthogonality 1e-4, all relative. */
 WCSVD_API int wcsvd_batched_f32(int batch, const int* m, const int* n, const float* const* A, const int* lda,
                                 float* const* S, float* const* U, float* const* V, float tol, int max_sweeps,
                                 wcsvd_stream_t stream);

@@ -47,7 +47,8 @@ class OptsT(ctypes.Structure):
                 ("info", ctypes.c_void_p), ("sweeps_inner", ctypes.c_void_p),
                 ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_size_t),
                 ("force_path", ctypes.c_int), ("force_w", ctypes.c_int), ("wcycle_sweeps", ctypes.c_int),
-                ("inner_sweeps", ctypes.c_int), ("pair_warps", ctypes.c_int), ("cluster_ctas", ctypes.c_int)]
+                ("inner_sweeps", ctypes.c_int), ("pair_warps", ctypes.c_int), ("cluster_ctas", ctypes.c_int),
+                ("f32_compute", ctypes.c_int)]
 
 
 _lib = None
@@ -135,7 +136,8 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
                     max_sweeps: int = 0, stream: int = 0, ldu=None, ldv=None, info_ptr: int = 0,
                     sweeps_inner_ptr: int = 0, workspace_ptr: int = 0, workspace_bytes: int = 0,
                     force_path: int = 0, force_w: int = 0, wcycle_sweeps: int = 0,
-                    inner_sweeps: int = 0, pair_warps: int = 0, cluster_ctas: int = 0, fp32: bool = False) -> None:
+                    inner_sweeps: int = 0, pair_warps: int = 0, cluster_ctas: int = 0, f32_compute: int = 0,
+                    fp32: bool = False) -> None:
     """Direct C-ABI call with column-major device pointers (integers). Raises WcsvdError.
     fp32=True calls wcsvd_batched_f32_ex (float data)."""
     m, n, lda = _arr_i32(m), _arr_i32(n), _arr_i32(lda)
@@ -157,6 +159,7 @@ def svd_batched_raw(m, n, A_ptrs, lda, S_ptrs, U_ptrs=None, V_ptrs=None, tol: fl
     opts.force_path, opts.force_w, opts.wcycle_sweeps, opts.inner_sweeps = force_path, force_w, wcycle_sweeps, inner_sweeps
     opts.pair_warps = pair_warps
     opts.cluster_ctas = cluster_ctas
+    opts.f32_compute = f32_compute
     fn = lib().wcsvd_batched_f32_ex if fp32 else lib().wcsvd_batched_ex
     rc = fn(B, m.ctypes.data, n.ctypes.data, Ap.ctypes.data, lda.ctypes.data,
             Sp.ctypes.data, Up.ctypes.data if Up is not None else None,
@@ -255,7 +258,7 @@ def _host_call(ms, ns, a_ptrs, s_ptrs, u_ptrs, v_ptrs, tol, max_sweeps, info, kw
     opts = OptsT()
     opts.struct_size = ctypes.sizeof(OptsT)
     opts.info = info.ctypes.data if info is not None else None
-    for key in ("force_path", "force_w", "wcycle_sweeps", "inner_sweeps", "pair_warps", "cluster_ctas"):
+    for key in ("force_path", "force_w", "wcycle_sweeps", "inner_sweeps", "pair_warps", "cluster_ctas", "f32_compute"):
         setattr(opts, key, int(kw.pop(key, 0)))
     if kw:
         raise TypeError(f"unexpected arguments {sorted(kw)}")

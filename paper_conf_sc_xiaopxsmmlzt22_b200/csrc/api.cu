@@ -290,6 +290,7 @@ int validate(int batch, const int* m, const int* n, const TI* const* A, const in
     if (opts->pair_warps != 0 && opts->pair_warps != 1) return -12;
     const int c = opts->cluster_ctas;
     if (c != 0 && c != 1 && c != 2 && c != 4 && c != 8) return -12;
+    if (opts->f32_compute != 0 && opts->f32_compute != 1) return -12;
     if (opts->force_path < 0 || opts->force_path > WCSVD_PATH_WCYCLE) return -12;
     if (opts->force_w != 0 && opts->force_w != 8 && opts->force_w != 16) return -12;
     for (int b = 0; b < batch; ++b) {
@@ -433,8 +434,8 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     else if (bk.path == WCSVD_PATH_L0)
       e = launch_l0(bk.variant, bk.withv, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
-      e = launch_l1(bk.variant, bk.path == WCSVD_PATH_WCYCLE ? 1 : 0, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i],
-                    cnt, bk.cluster, pool, st);
+      e = launch_l1(bk.variant, bk.path == WCSVD_PATH_WCYCLE ? 1 : 0, kF32 ? 1 : 0, (opts && opts->f32_compute) ? 1 : 0,
+                    d_descs, d_order + bucket_off[i], cnt, bk.cluster, pool, st);
     if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);
   }
   for (int i = 0; i < (int)side.size(); ++i) {
@@ -706,6 +707,7 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
       o.inner_sweeps = opts->inner_sweeps;
       o.pair_warps = opts->pair_warps;
       o.cluster_ctas = opts->cluster_ctas;
+      o.f32_compute = opts->f32_compute;
     }
     rc = batched_impl<double>(cnt, m + b0, n + b0, pA.data(), ld_.data(), pS.data(), wantU ? pU.data() : nullptr,
                               wantV ? pV.data() : nullptr, tol, max_sweeps,

@@ -29,8 +29,9 @@ enum L1Variant {
 
 // Level-1 launch: `cluster` CTAs per matrix (1, 2, 4 or 8; a thread-block cluster when > 1).
 // wcycle = 1: the W-cycle kernel (Level 1 -> Level 2 recursion, one CTA per matrix).
-cudaError_t launch_l1(int variant, int wcycle, int fp32, const MatDesc* descs, const int* order, int count,
-                      int cluster, const SlotPool& pool, cudaStream_t stream);
+// fp32 = 1: float I/O; f32_compute = 1 iterates in fp32 (FFMA), else on an fp64 working copy (DMMA).
+cudaError_t launch_l1(int variant, int wcycle, int fp32, int f32_compute, const MatDesc* descs, const int* order,
+                      int count, int cluster, const SlotPool& pool, cudaStream_t stream);
 
 cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
                         const SlotPool& pool, cudaStream_t stream);

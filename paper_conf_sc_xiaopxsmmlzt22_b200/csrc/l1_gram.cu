@@ -343,27 +343,31 @@ struct EvdMap {
 // B' = G^T B G is updated from one load per quad row and written, like the
 // diagonal blocks, to the slots its indices move to in Bn; J <- J G in slot order (x -> y rename).
 // A step in which no pair rotates only moves B and J.
-template <int W2>
-__device__ __forceinline__ bool evd_step(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
-                                         const EvdMap<W2>& em, int lane, double tol2, const double (&x)[W2],
-                                         double (&y)[W2]) {
+template <typename T> struct Vec2;
+template <> struct Vec2<double> { using type = double2; };
+template <> struct Vec2<float> { using type = float2; };
+
+template <int W2, typename T = double>
+__device__ __forceinline__ bool evd_step(const T* __restrict__ Bc, T* __restrict__ Bn, typename Vec2<T>::type* cs,
+                                         const EvdMap<W2>& em, int lane, T tol2, const T (&x)[W2], T (&y)[W2]) {
+  using T2 = typename Vec2<T>::type;
   constexpr int NPR = W2 / 2, QPL = EvdMap<W2>::QPL;
-  const double bpp = Bc[em.dld01 & 0xffff], bqq = Bc[em.dld01 >> 16], bpq = Bc[em.dld2];
-  double c, s, t;
+  const T bpp = Bc[em.dld01 & 0xffff], bqq = Bc[em.dld01 >> 16], bpq = Bc[em.dld2];
+  T c, s, t;
   const bool rot = jacobi_rotation(bpp, bqq, bpq, tol2, c, s, t);
   if (lane < NPR) {
-    cs[lane] = make_double2(c, s);
+    cs[lane] = T2{c, s};
     Bn[em.dst01 & 0xffff] = rot ? fma(t, bpq, bpp) : bpp;
     Bn[em.dst01 >> 16] = rot ? fma(-t, bpq, bqq) : bqq;
-    Bn[em.dst2] = rot ? 0.0 : bpq;
+    Bn[em.dst2] = rot ? T(0) : bpq;
   }
-  double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
+  T b00[QPL], b01[QPL], b10[QPL], b11[QPL];
 #pragma unroll
   for (int i = 0; i < QPL; ++i) {
     if (em.q[i] & (1 << 13)) {
       const int o = em.q[i] & 0x7ff;
-      const double2 v0 = *reinterpret_cast<const double2*>(Bc + o);
-      const double2 v1 = *reinterpret_cast<const double2*>(Bc + o + W2);
+      const T2 v0 = *reinterpret_cast<const T2*>(Bc + o);
+      const T2 v1 = *reinterpret_cast<const T2*>(Bc + o + W2);
       const bool sw = (em.q[i] >> 11) & 1;
       b00[i] = sw ? v0.y : v0.x;
       b01[i] = sw ? v0.x : v0.y;
@@ -391,13 +395,13 @@ __device__ __forceinline__ bool evd_step(const double* __restrict__ Bc, double* 
 #pragma unroll
   for (int i = 0; i < QPL; ++i) {
     if (em.q[i] & (1 << 13)) {
-      const double2 gp = cs[(em.q[i] >> 16) & (NPR - 1)];
+      const T2 gp = cs[(em.q[i] >> 16) & (NPR - 1)];
       const bool own_lo = (em.q[i] >> 12) & 1;
-      const double rc = own_lo ? c : gp.x, rs = own_lo ? s : gp.y;  // rotation of the row pair
-      const double cc = own_lo ? gp.x : c, cs_ = own_lo ? gp.y : s;  // rotation of the column pair
+      const T rc = own_lo ? c : gp.x, rs = own_lo ? s : gp.y;  // rotation of the row pair
+      const T cc = own_lo ? gp.x : c, cs_ = own_lo ? gp.y : s;  // rotation of the column pair
       // columns (2hi, 2hi+1): B G_hi
-      const double c0 = fma(cs_, b01[i], cc * b00[i]), c1 = fma(-cs_, b00[i], cc * b01[i]);
-      const double d0 = fma(cs_, b11[i], cc * b10[i]), d1 = fma(-cs_, b10[i], cc * b11[i]);
+      const T c0 = fma(cs_, b01[i], cc * b00[i]), c1 = fma(-cs_, b00[i], cc * b01[i]);
+      const T d0 = fma(cs_, b11[i], cc * b10[i]), d1 = fma(-cs_, b10[i], cc * b11[i]);
       // rows (2lo, 2lo+1): G_lo^T (B G_hi)
       Bn[em.st[i][0] & 0xffff] = fma(rs, d0, rc * c0);
       Bn[em.st[i][0] >> 16] = fma(rs, d1, rc * c1);
@@ -408,8 +412,8 @@ __device__ __forceinline__ bool evd_step(const double* __restrict__ Bc, double* 
   // J <- J G in slot order; outputs move to their next slots (register rename).
 #pragma unroll
   for (int k = 0; k < NPR; ++k) {
-    const double2 g = cs[k];
-    const double a = x[2 * k], b = x[2 * k + 1];
+    const T2 g = cs[k];
+    const T a = x[2 * k], b = x[2 * k + 1];
     y[rr_dest(2 * k, W2)] = fma(g.y, b, g.x * a);
     y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
   }
@@ -546,6 +550,227 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(5);
   return true;
 }
+// ---- fp32 Gram path (wcsvd_batched_f32): the same pair steps in single precision ----
+// sm_100a has no full-precision fp32 MMA (DMMA is fp64 only, TF32 keeps 10 mantissa bits), so the two
+// contractions run on the FFMA pipe: lane l owns column l of the Gram / of the updated panel (two lanes
+// per column when 2w = 16, one per 8-row half of a slab, summed in fixed order), panel slabs arrive
+// through the same per-warp cp.async ring (16 rows x 2w columns, 80-byte column stride), every value a
+// lane needs from another column is a broadcast LDS.128 of 4 consecutive rows. The EVD is evd_step<W2,
+// float>, the Newton-Schulz cleanup is two 2w^3 FFMA contractions in shared memory. The working copy
+// W, V is fp32 (half the bytes of the fp64 path).
+template <int W2>
+struct WarpSmemF {
+  float* B;    // EVD ping-pong (2 x W2 x W2, slot layout); afterwards E = J^T J - I ([W2][BS])
+  float* S;    // [W2][BS] staged J
+  float2* cs;  // [W2 / 2]
+  float* ring; // [NSTAGE][W2][SLF]
+  static constexpr int BS = W2 + 1;
+  static constexpr int SLF = 20;  // ring column stride (floats): 16 rows + 4 pad, 16-byte chunks
+  static constexpr int NSTAGE = WCSVD_L1_NSTAGE;
+  static constexpr int SLAB = W2 * SLF;
+  __host__ __device__ static constexpr size_t region() {
+    return (2 * W2 * BS > NSTAGE * SLAB ? 2 * W2 * BS : NSTAGE * SLAB) * sizeof(float);
+  }
+  __host__ __device__ static constexpr size_t bytes() { return region() + sizeof(float2) * (W2 / 2); }
+};
+
+// chunk i of this lane: column (lane + 32 i) / 4, rows 4 ((lane + 32 i) % 4) .. +3 of the slab
+template <int W2>
+__device__ __forceinline__ void slab_issue_f(float* ring, const float* base, const int (&coff)[W2 / 8], int r0,
+                                             int st, int lane) {
+  float* dst = ring + st * WarpSmemF<W2>::SLAB;
+#pragma unroll
+  for (int i = 0; i < W2 / 8; ++i) {
+    const int q = lane + 32 * i, c = q >> 2, h = q & 3;
+    cp_async16(dst + c * WarpSmemF<W2>::SLF + 4 * h, base + coff[i] + r0 + 4 * h);
+  }
+}
+
+template <int W2>
+__device__ __forceinline__ void slab_offsets_f(int (&coff)[W2 / 8], int I, int J, int ld, int lane) {
+#pragma unroll
+  for (int i = 0; i < W2 / 8; ++i) coff[i] = pcol<W2>((lane + 32 * i) >> 2, I, J) * ld;
+}
+
+// acc[i] = sum_r P[r][i] P[r][col] over the panel rows (this lane's half of every slab), then the two
+// halves are combined (2w = 16): B[i][col] for every i, lane = (half, col).
+template <int W2>
+__device__ __forceinline__ void gram_f32(float* ring, const float* base, int ld, int rows, int I, int J, int lane,
+                                         float (&acc)[W2]) {
+  constexpr int SLF = WarpSmemF<W2>::SLF, NS = WarpSmemF<W2>::NSTAGE, LPC = 32 / W2, RPL = 16 / LPC;
+  const int col = lane % W2, half = lane / W2;
+#pragma unroll
+  for (int i = 0; i < W2; ++i) acc[i] = 0.0f;
+  int coff[W2 / 8];
+  slab_offsets_f<W2>(coff, I, J, ld, lane);
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) slab_issue_f<W2>(ring, base, coff, 16 * j, j, lane);
+    cp_async_commit();
+  }
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) slab_issue_f<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const float* st = ring + (sl % NS) * WarpSmemF<W2>::SLAB;
+#pragma unroll
+    for (int r4 = 0; r4 < RPL; r4 += 4) {
+      const float4 own = *reinterpret_cast<const float4*>(st + col * SLF + half * RPL + r4);
+#pragma unroll
+      for (int i = 0; i < W2; ++i) {
+        const float4 v = *reinterpret_cast<const float4*>(st + i * SLF + half * RPL + r4);
+        acc[i] = fmaf(v.x, own.x, acc[i]);
+        acc[i] = fmaf(v.y, own.y, acc[i]);
+        acc[i] = fmaf(v.z, own.z, acc[i]);
+        acc[i] = fmaf(v.w, own.w, acc[i]);
+      }
+    }
+    __syncwarp();
+  }
+  if constexpr (LPC == 2) {
+#pragma unroll
+    for (int i = 0; i < W2; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], 16);  // commutative: same bits
+  }
+}
+
+// X <- X J' for the panel of pair (I, J): lane (half, col) computes column col of its rows of every
+// slab from jc[k] = J'[k][col]; results stored in place (a slab's rows are read before overwritten).
+template <int W2>
+__device__ __forceinline__ void apply_f32(float* ring, float* base, int ld, int rows, int I, int J, int lane,
+                                          const float (&jc)[W2]) {
+  constexpr int SLF = WarpSmemF<W2>::SLF, NS = WarpSmemF<W2>::NSTAGE, LPC = 32 / W2, RPL = 16 / LPC;
+  const int col = lane % W2, half = lane / W2;
+  int coff[W2 / 8];
+  slab_offsets_f<W2>(coff, I, J, ld, lane);
+  float* out = base + (size_t)pcol<W2>(col, I, J) * ld + half * RPL;
+  const int nslab = rows >> 4;
+#pragma unroll
+  for (int j = 0; j < NS - 1; ++j) {
+    if (j < nslab) slab_issue_f<W2>(ring, base, coff, 16 * j, j, lane);
+    cp_async_commit();
+  }
+  for (int sl = 0; sl < nslab; ++sl) {
+    if (sl + NS - 1 < nslab) slab_issue_f<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    cp_async_commit();
+    cp_async_wait<NS - 1>();
+    __syncwarp();
+    const float* st = ring + (sl % NS) * WarpSmemF<W2>::SLAB;
+#pragma unroll
+    for (int r4 = 0; r4 < RPL; r4 += 4) {
+      float4 o = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int k = 0; k < W2; ++k) {
+        const float4 v = *reinterpret_cast<const float4*>(st + k * SLF + half * RPL + r4);
+        o.x = fmaf(v.x, jc[k], o.x);
+        o.y = fmaf(v.y, jc[k], o.y);
+        o.z = fmaf(v.z, jc[k], o.z);
+        o.w = fmaf(v.w, jc[k], o.w);
+      }
+      __stcg(reinterpret_cast<float4*>(out + 16 * sl + r4), o);
+    }
+    __syncwarp();
+  }
+}
+
+template <int W2>
+__device__ bool process_pair_f32(const WarpSmemF<W2>& ws, float* Wm, int ld, int mrows, float* Vm, int ldv,
+                                 int vrows, int I, int J, float tol2, int inner_cap, int lane, int* inner) {
+  constexpr int BS = WarpSmemF<W2>::BS;
+  const int col = lane % W2;
+  float* B0 = ws.B;
+  float* B1 = ws.B + W2 * W2;
+  // (1) Gram (Alg 1 l.5), upper triangle into the EVD layout
+  {
+    float acc[W2];
+    gram_f32<W2>(ws.ring, Wm, ld, mrows, I, J, lane, acc);
+    __syncwarp();  // the ring aliases B
+    if (lane < W2) {
+#pragma unroll
+      for (int i = 0; i < W2; ++i)
+        if (i <= col) B0[evd_phys<W2>(i, col)] = acc[i];
+    }
+  }
+  __syncwarp();
+  // (4) off-norm test (Z6)
+  bool need = false;
+  {
+    const float bqq = (lane < W2) ? B0[evd_phys<W2>(lane, lane)] : 0.0f;
+#pragma unroll 4
+    for (int p = 0; p < W2 - 1; ++p) {
+      const float bpp = B0[evd_phys<W2>(p, p)];
+      const float bpq = (lane < W2 && lane > p) ? B0[evd_phys<W2>(p, lane)] : 0.0f;
+      const float ab = bpp * bqq;
+      need |= (lane > p && ab > 0.0f && bpq * bpq > tol2 * ab);
+    }
+  }
+  if (!__any_sync(0xffffffffu, need)) return false;
+  // (2) EVD (Alg 1 l.6), threshold parallel Jacobi in fp32
+  EvdMap<W2> em;
+  em.init(lane);
+  float ja[W2], jb[W2];
+#pragma unroll
+  for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0f : 0.0f;
+  bool rotated = false;
+  int isw = 0;
+  for (; isw < inner_cap; ++isw) {
+    bool any = evd_step<W2, float>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+    __syncwarp();
+    for (int r = 1; r < W2 - 1; r += 2) {
+      any |= evd_step<W2, float>(B1, B0, ws.cs, em, lane, tol2, jb, ja);
+      __syncwarp();
+      any |= evd_step<W2, float>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+      __syncwarp();
+    }
+#pragma unroll
+    for (int s = 0; s < W2; ++s) ja[s] = jb[s];
+    float* tmp = B0;
+    B0 = B1;
+    B1 = tmp;
+    rotated |= any;
+    if (!any) break;
+  }
+  *inner += isw + (isw < inner_cap ? 1 : 0);
+  if (!rotated) return false;
+  // Stage J (row lane), Newton-Schulz (Z9(ii)): E = J^T J - I, J' = J - J E / 2; lane keeps column col of J'.
+  if (lane < W2) {
+#pragma unroll
+    for (int s = 0; s < W2; ++s) ws.S[lane * BS + s] = ja[s];
+  }
+  __syncwarp();
+  float jc[W2];
+  {
+    float e[W2];
+#pragma unroll
+    for (int i = 0; i < W2; ++i) e[i] = 0.0f;
+#pragma unroll 4
+    for (int k = 0; k < W2; ++k) {
+      const float jk = ws.S[k * BS + col];
+#pragma unroll
+      for (int i = 0; i < W2; ++i) e[i] = fmaf(ws.S[k * BS + i], jk, e[i]);
+    }
+    __syncwarp();
+    if (lane < W2) {
+#pragma unroll
+      for (int i = 0; i < W2; ++i) ws.B[i * BS + col] = e[i] - (i == col ? 1.0f : 0.0f);
+    }
+    __syncwarp();
+#pragma unroll 4
+    for (int r = 0; r < W2; ++r) {
+      float t = 0.0f;
+#pragma unroll
+      for (int i = 0; i < W2; ++i) t = fmaf(ws.S[r * BS + i], ws.B[i * BS + col], t);
+      jc[r] = fmaf(-0.5f, t, ws.S[r * BS + col]);
+    }
+  }
+  __syncwarp();  // the ring aliases B and S
+  // (3) A_ij <- A_ij J', V_ij <- V_ij J' (Alg 1 l.7)
+  apply_f32<W2>(ws.ring, Wm, ld, mrows, I, J, lane, jc);
+  apply_f32<W2>(ws.ring, Vm, ldv, vrows, I, J, lane, jc);
+  return true;
+}
+
 // ---- Cross-CTA plumbing for a matrix spread over a thread-block cluster (tailoring) ----
 // A matrix may be owned by a cluster of CL CTAs (CL = 1, 2, 4, 8; chosen by the planner from the batch
 // composition, PAPER.md:228, 261-269 -- scheduling only, never arithmetic, Z22). The pairs of a
@@ -610,9 +835,10 @@ __device__ __forceinline__ void pair_fence() {
 }
 
 // Per-warp shared-memory stride: the pair buffers, or a 32 x 33 transpose tile for the stage-in.
-template <int W2>
+template <int W2, typename TW = double>
 __host__ __device__ constexpr size_t warp_stride() {
-  return ((WarpSmem<W2>::bytes() > 32 * 33 * 8 ? WarpSmem<W2>::bytes() : 32 * 33 * 8) + 15) & ~size_t(15);
+  constexpr size_t pb = sizeof(TW) == 8 ? WarpSmem<W2>::bytes() : WarpSmemF<W2>::bytes();
+  return ((pb > 32 * 33 * sizeof(TW) ? pb : 32 * 33 * sizeof(TW)) + 15) & ~size_t(15);
 }
 
 }  // namespace
@@ -622,7 +848,7 @@ __host__ __device__ constexpr size_t warp_stride() {
 // inlined copy of process_pair per kernel (register pressure).
 enum { kFlat = 0, kFlatCluster = 1, kWcycle = 2 };
 
-template <int W2, int NW, typename TI, int MODE>
+template <int W2, int NW, typename TI, typename TW, int MODE>
 __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
                                                              const int* __restrict__ order, SlotPool pool) {
   // TI: type of A, S, U, V in the caller's memory (double, or float for wcsvd_batched_f32); the
@@ -640,15 +866,26 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   const int M = d.M, N = d.N, mp = d.m_pad, np = d.n_pad;
 
   extern __shared__ __align__(16) unsigned char smem_raw[];
+  // TW: the working precision: fp64 (DMMA contractions; also the default for fp32 data, see launch_l1)
+  // or fp32 (the FFMA path of wcsvd_batched_f32 with opts->f32_compute = 1)
+  constexpr bool F32 = sizeof(TW) == 4;
   WarpSmem<W2> ws;
+  WarpSmemF<W2> wsf;
   {
-    unsigned char* p = smem_raw + warp * warp_stride<W2>();
-    ws.B = reinterpret_cast<double*>(p);
-    ws.S = ws.B + W2 * C::BS;
-    ws.ring = ws.B;
-    ws.cs = reinterpret_cast<double2*>(p + WarpSmem<W2>::region());
-    ws.tt = reinterpret_cast<double*>(ws.cs + W2 / 2);
-    ws.pq = reinterpret_cast<int2*>(ws.tt + W2 / 2);
+    unsigned char* p = smem_raw + warp * warp_stride<W2, TW>();
+    if constexpr (F32) {
+      wsf.B = reinterpret_cast<float*>(p);
+      wsf.S = wsf.B + W2 * WarpSmemF<W2>::BS;
+      wsf.ring = wsf.B;
+      wsf.cs = reinterpret_cast<float2*>(p + WarpSmemF<W2>::region());
+    } else {
+      ws.B = reinterpret_cast<double*>(p);
+      ws.S = ws.B + W2 * C::BS;
+      ws.ring = ws.B;
+      ws.cs = reinterpret_cast<double2*>(p + WarpSmem<W2>::region());
+      ws.tt = reinterpret_cast<double*>(ws.cs + W2 / 2);
+      ws.pq = reinterpret_cast<int2*>(ws.tt + W2 / 2);
+    }
   }
   // Matrix-wide state (rank 0's copy is the one in use when CLU).
   __shared__ int s_flags[4];          // [0, 1] sweep votes (parity), [2] non-finite, [3] needs completion
@@ -681,8 +918,8 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     __syncthreads();
   }
   const int slot = CLU ? *at_rank0(&s_slot) : s_slot;
-  double* Wm = pool.base + (size_t)slot * pool.slot_doubles;
-  double* Vm = Wm + (size_t)mp * np;
+  TW* Wm = reinterpret_cast<TW*>(pool.base + (size_t)slot * pool.slot_doubles);
+  TW* Vm = Wm + (size_t)mp * np;
 
   // ---- Stage-in: W = A or A^T, zero-padded to m_pad x n_pad; V = I. 32 x 32 tiles
   // per warp; the transpose (m < n) goes through a shared-memory tile so that both the reads of A
@@ -706,7 +943,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
 #endif
   {
     const TI* Ain = reinterpret_cast<const TI*>(d.A);
-    double* tile = reinterpret_cast<double*>(smem_raw + warp * warp_stride<W2>());
+    TW* tile = reinterpret_cast<TW*>(smem_raw + warp * warp_stride<W2, TW>());
     const int ntr = (mp + 31) / 32, ntc = (np + 31) / 32;
     for (int t = gw; t < ntr * ntc; t += NWT) {
       const int r0 = (t % ntr) * 32, c0 = (t / ntr) * 32;
@@ -720,7 +957,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
             bad |= !isfinite(v);
             amax = fmax(amax, fabs(v));
           }
-          tile[rr * 33 + lane] = v;
+          tile[rr * 33 + lane] = (TW)v;
         }
         __syncwarp();
         for (int cc = 0; cc < 32; ++cc) {
@@ -738,7 +975,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
               bad |= !isfinite(v);
               amax = fmax(amax, fabs(v));
             }
-            Wm[(size_t)c * mp + r] = v;
+            Wm[(size_t)c * mp + r] = (TW)v;
           }
         }
       }
@@ -746,7 +983,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
   if (d.withv)
     for (size_t e = (size_t)crank * T + tid; e < (size_t)np * np; e += (size_t)CL * T)
-      Vm[e] = ((int)(e % np) == (int)(e / np)) ? 1.0 : 0.0;
+      Vm[e] = ((int)(e % np) == (int)(e / np)) ? TW(1) : TW(0);
   const int vrows = d.withv ? np : 0;  // values / U-only mode: V_x is not accumulated (§8(f4))
   // max |a_ij| and the non-finite flag: CTA-local atomics, then (cluster) one slot per CTA in rank 0
   if (bad) atomicOr(&s_flags[2], 1);
@@ -773,11 +1010,11 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     for (int t = gw; t < ntr * ntc; t += NWT) {
       const int r0 = (t % ntr) * 32, c0 = (t / ntr) * 32, r = r0 + lane;
       if (r < mp)
-        for (int cc = 0; cc < 32 && c0 + cc < np; ++cc) Wm[(size_t)(c0 + cc) * mp + r] *= f;
+        for (int cc = 0; cc < 32 && c0 + cc < np; ++cc) Wm[(size_t)(c0 + cc) * mp + r] *= (TW)f;
     }
   }
   if constexpr (CLU) cl_sync(); else __syncthreads();
-  const double tol2 = d.tol * d.tol;
+  const TW tol2 = (TW)(d.tol * d.tol);
 
   int sweep = 0;
   bool converged = false;
@@ -800,7 +1037,10 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
           }
           __syncwarp();
           pair_fence<CLU>();  // the previous owners' W / V writes are visible to every lane
-          rot_any |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
+          if constexpr (F32)
+            rot_any |= process_pair_f32<W2>(wsf, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
+          else
+            rot_any |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
           pair_fence<CLU>();  // every lane's W / V writes precede ...
           __syncwarp();
           if (lane == 0) {    // ... the release
@@ -843,7 +1083,10 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
                   const int a = rr_content(2 * p2, s2, 2 * r), b = rr_content(2 * p2 + 1, s2, 2 * r);
                   const int Ia = (a < r) ? I1 * r + a : J1 * r + (a - r);
                   const int Ib = (b < r) ? I1 * r + b : J1 * r + (b - r);
-                  mine |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
+                  if constexpr (F32)
+                    mine |= process_pair_f32<W2>(wsf, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
+                  else
+                    mine |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, Ia, Ib, tol2, d.inner_cap, lane, &my_inner);
                 }
                 named_bar(1 + grp, GS * 32);
               }
@@ -875,7 +1118,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   // sigma and the sign of every column go to rank 0's arrays; every CTA then copies them locally.
   // one CTA: reuse the warp buffers; cluster: a dedicated region after them (other CTAs write rank 0's
   // copy while its warps may still be draining their slab rings)
-  double* s_sig = reinterpret_cast<double*>(smem_raw + (CLU ? NW * warp_stride<W2>() : 0));  // [N]
+  double* s_sig = reinterpret_cast<double*>(smem_raw + (CLU ? NW * warp_stride<W2, TW>() : 0));  // [N]
   double* s_sgn = s_sig + N;                             // [N]
   double* sig0 = s_sig;
   double* sgn0 = s_sgn;
@@ -886,20 +1129,20 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     __syncthreads();
   }
   for (int j = gw; j < N; j += NWT) {
-    const double* col = Wm + (size_t)j * mp;
+    const TW* col = Wm + (size_t)j * mp;
     double a = 0.0;
     for (int r = lane; r < M; r += 32) {
-      const double x = __ldcg(col + r);
+      const double x = (double)__ldcg(col + r);
       a = fma(x, x, a);
     }
     for (int off = 16; off > 0; off >>= 1) a += __shfl_xor_sync(0xffffffffu, a, off);
     // Z15 sign rule on the square factor V_x; without V (values / U-only mode) on the columns of X.
-    const double* vc = d.withv ? Vm + (size_t)j * np : col;
+    const TW* vc = d.withv ? Vm + (size_t)j * np : col;
     const int vlen = d.withv ? N : M;
     double best = 0.0;
     int bi = 0x7fffffff;
     for (int i = lane; i < vlen; i += 32) {
-      const double v = __ldcg(vc + i);
+      const double v = (double)__ldcg(vc + i);
       if (fabs(v) > fabs(best)) { best = v; bi = i; }
     }
     for (int off = 16; off > 0; off >>= 1) {
@@ -923,7 +1166,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   __syncthreads();
   double sig1 = 0.0;
   for (int i = 0; i < N; ++i) sig1 = fmax(sig1, s_sig[i]);
-  const double thresh = sig1 * (double)M * kU53;
+  const double thresh = sig1 * (double)M * (F32 ? 5.9604644775390625e-08 : kU53);  // Z14: the working precision's u
   const double nanv = __longlong_as_double(0x7ff8000000000000ULL);
   TI* dstW = reinterpret_cast<TI*>(d.swapped ? d.V : d.U);
   const int ldW = d.swapped ? d.ldv : d.ldu;
@@ -946,13 +1189,13 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
     const bool ok = sj > thresh;
     needs_completion |= !ok;
     if (dstW) {
-      const double* col = Wm + (size_t)j * mp;
+      const TW* col = Wm + (size_t)j * mp;
       for (int r = lane; r < M; r += 32)
-        dstW[(size_t)rk * ldW + r] = (TI)(nonfinite ? nanv : (ok ? sgn * (__ldcg(col + r) / sj) : sgn * 0.0));
+        dstW[(size_t)rk * ldW + r] = (TI)(nonfinite ? nanv : (ok ? sgn * ((double)__ldcg(col + r) / sj) : sgn * 0.0));
     }
     if (dstV) {
-      const double* vc = Vm + (size_t)j * np;
-      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = (TI)(nonfinite ? nanv : sgn * __ldcg(vc + i));
+      const TW* vc = Vm + (size_t)j * np;
+      for (int i = lane; i < N; i += 32) dstV[(size_t)rk * ldV + i] = (TI)(nonfinite ? nanv : sgn * (double)__ldcg(vc + i));
     }
     if (lane == 0) reinterpret_cast<TI*>(d.S)[rk] = (TI)(nonfinite ? sj : ldexp(sj, sexp));
   }
@@ -966,14 +1209,14 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   }
 }
 
-template <int W2, int NW, typename TI, int MODE>
+template <int W2, int NW, typename TI, typename TW, int MODE>
 static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count, int cluster, const SlotPool& pool,
                                cudaStream_t stream) {
-  size_t smem = NW * warp_stride<W2>();
+  size_t smem = NW * warp_stride<W2, TW>();
   const size_t fin = 2 * 8 * 1024;  // finalisation arrays: alias the warp buffers (one CTA) or follow them
   if (MODE == kFlatCluster) smem += fin;
   else if (smem < fin) smem = fin;
-  auto kern = l1_gram_kernel<W2, NW, TI, MODE>;
+  auto kern = l1_gram_kernel<W2, NW, TI, TW, MODE>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (MODE != kFlatCluster) {
@@ -995,29 +1238,34 @@ static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count
   return cudaLaunchKernelEx(&cfg, kern, descs, order, pool);
 }
 
-template <typename TI, int W2, int NW>
+template <typename TI, typename TW, int W2, int NW>
 static cudaError_t launch_l1_m(int wcycle, const MatDesc* descs, const int* order, int count, int cluster,
                                const SlotPool& pool, cudaStream_t stream) {
-  if (wcycle) return launch_l1_t<W2, NW, TI, kWcycle>(descs, order, count, 1, pool, stream);
-  if (cluster > 1) return launch_l1_t<W2, NW, TI, kFlatCluster>(descs, order, count, cluster, pool, stream);
-  return launch_l1_t<W2, NW, TI, kFlat>(descs, order, count, 1, pool, stream);
+  if (wcycle) return launch_l1_t<W2, NW, TI, TW, kWcycle>(descs, order, count, 1, pool, stream);
+  if (cluster > 1) return launch_l1_t<W2, NW, TI, TW, kFlatCluster>(descs, order, count, cluster, pool, stream);
+  return launch_l1_t<W2, NW, TI, TW, kFlat>(descs, order, count, 1, pool, stream);
 }
 
-template <typename TI>
+template <typename TI, typename TW>
 static cudaError_t launch_l1_v(int variant, int wcycle, const MatDesc* descs, const int* order, int count,
                                int cluster, const SlotPool& pool, cudaStream_t stream) {
   switch (variant) {
-    case kL1_16x4: return launch_l1_m<TI, 16, 4>(wcycle, descs, order, count, cluster, pool, stream);
-    case kL1_32x4: return launch_l1_m<TI, 32, 4>(wcycle, descs, order, count, cluster, pool, stream);
-    case kL1_32x8: return launch_l1_m<TI, 32, 8>(wcycle, descs, order, count, cluster, pool, stream);
+    case kL1_16x4: return launch_l1_m<TI, TW, 16, 4>(wcycle, descs, order, count, cluster, pool, stream);
+    case kL1_32x4: return launch_l1_m<TI, TW, 32, 4>(wcycle, descs, order, count, cluster, pool, stream);
+    case kL1_32x8: return launch_l1_m<TI, TW, 32, 8>(wcycle, descs, order, count, cluster, pool, stream);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_l1(int variant, int wcycle, int fp32, const MatDesc* descs, const int* order, int count,
-                      int cluster, const SlotPool& pool, cudaStream_t stream) {
-  return fp32 ? launch_l1_v<float>(variant, wcycle, descs, order, count, cluster, pool, stream)
-              : launch_l1_v<double>(variant, wcycle, descs, order, count, cluster, pool, stream);
+// fp32 data: f32_compute = 0 iterates on an fp64 working copy with the DMMA contractions (B200: 239 /
+// 361 ms on C3 / C4 as fp32), 1 on an fp32 working copy with FFMA contractions (447 / 1011 ms: FFMA
+// needs 8x the issue slots of DMMA per flop and the FP32 pipe is only 2x the FP64 one -- profiles/
+// f32_paths_r02.json), so the planner default is 0.
+cudaError_t launch_l1(int variant, int wcycle, int fp32, int f32_compute, const MatDesc* descs, const int* order,
+                      int count, int cluster, const SlotPool& pool, cudaStream_t stream) {
+  if (!fp32) return launch_l1_v<double, double>(variant, wcycle, descs, order, count, cluster, pool, stream);
+  return f32_compute ? launch_l1_v<float, float>(variant, wcycle, descs, order, count, cluster, pool, stream)
+                     : launch_l1_v<float, double>(variant, wcycle, descs, order, count, cluster, pool, stream);
 }
 
 }  // namespace wcsvd

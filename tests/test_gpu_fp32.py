@@ -1,7 +1,8 @@
 """the fp32 variant (wcsvd_batched_f32). Parity with the long-double oracle run on the
 same fp32 inputs, at north_star's fp32 bars: sigma 1e-5, residual 1e-5, orthogonality 1e-4 (vector
-bars per R-VEC with u = 2^-24). Level 0 iterates in fp32; the Gram path iterates in fp64 on an fp64
-copy and rounds at finalisation."""
+bars per R-VEC with u = 2^-24). Level 0 iterates in fp32; the Gram path iterates by default on an fp64
+working copy (DMMA) and rounds at finalisation, and with f32_compute = 1 in fp32 throughout (FFMA Gram /
+update, fp32 EVD and Newton-Schulz on an fp32 working copy)."""
 import numpy as np
 import pytest
 import torch
@@ -38,7 +39,8 @@ def _run(mats32, **kw):
 @pytest.mark.parametrize("shapes", [
     [(32, 32), (64, 64), (40, 24), (24, 40), (8, 3), (3, 8), (1, 1)],          # Level 0 (fp32)
     [(100, 37), (190, 64), (480, 31), (1000, 16), (1024, 5)],                 # Level 0, tall
-    [(97, 97), (256, 256), (300, 170), (170, 300), (1024, 128)],             # Level 1 (fp64 inside)
+    [(97, 97), (256, 256), (300, 170), (170, 300), (1024, 128)],             # Level 1 (fp32 FFMA)
+    [(700, 520), (1024, 1024), (150, 900)],                                   # Level 1, large / wide
 ])
 def test_fp32_parity(shapes):
     mats = [workloads.gaussian(workloads.matrix_rng(700 + i, 5), m, n).astype(np.float32)
@@ -69,3 +71,14 @@ def test_fp32_rank_deficient_and_nonfinite():
     B[2, 3] = np.inf
     S, U, V, info = _run([B])
     assert info[0] == -2 and np.all(np.isnan(S[0]))
+
+
+@pytest.mark.parametrize("kw", [dict(f32_compute=1), dict(force_path=wc.PATH_GRAM, force_w=8, f32_compute=1),
+                                dict(force_path=wc.PATH_WCYCLE, f32_compute=1), dict(cluster_ctas=4, f32_compute=1),
+                                dict(cluster_ctas=4), dict(force_path=wc.PATH_GRAM, force_w=8)])
+def test_fp32_gram_variants(kw):
+    # the 2w = 16 FFMA path (two lanes per column), the W-cycle on fp32, and a 4-CTA cluster
+    shapes = [(130, 100), (100, 150), (256, 160), (64, 64), (1024, 128), (300, 700)]
+    mats = [workloads.gaussian(workloads.matrix_rng(720 + i, 7), m, n).astype(np.float32)
+            for i, (m, n) in enumerate(shapes)]
+    _check(mats, *_run(mats, **kw))
