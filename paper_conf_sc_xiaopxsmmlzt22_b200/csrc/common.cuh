@@ -39,6 +39,14 @@ WCSVD_HD int rr_dest(int slot, int np) {
   if (r == L) r = 0;
   return rr_slot_of_ring(r, np);
 }
+// Slot whose value moves into `slot` after one step (inverse of rr_dest).
+WCSVD_HD int rr_src(int slot, int np) {
+  if (slot == 0 || np == 2) return slot;
+  const int L = np - 1;
+  int r = rr_ring_index(slot, np) - 1;
+  if (r < 0) r += L;
+  return rr_slot_of_ring(r, np);
+}
 // Original index held by `slot` at step s (0 <= s < np-1).
 WCSVD_HD int rr_content(int slot, int s, int np) {
   if (slot == 0 || np == 2) return slot;

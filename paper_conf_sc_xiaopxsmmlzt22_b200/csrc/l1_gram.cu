@@ -464,13 +464,14 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_COUNT(7);
   if (!__any_sync(0xffffffffu, need)) return false;
   // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, B and J in slot order.
-  EvdMap<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
-  em.init(lane);
   double ja[W2], jb[W2];
-#pragma unroll
-  for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
   bool rotated = false;
   int isw = 0;
+  {
+  EvdMap<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
+  em.init(lane);
+#pragma unroll
+  for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
   for (; isw < inner_cap; ++isw) {
     // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb / B1, slots back in order.
     bool any = evd_step<W2>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
@@ -488,6 +489,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
     B1 = tmp;
     rotated |= any;
     if (!any) break;
+  }
   }
   *inner += isw + (isw < inner_cap ? 1 : 0);
   PHASE_MARK(2);

@@ -1,5 +1,4 @@
-"""Small mixed batch for compute-sanitizer runs (L0 variants, L1 flat w=8/16, W-cycle, the split pair
-executor, the host-buffer pipeline)."""
+"""Small mixed batch for compute-sanitizer runs (L0 variants, L1 flat w=8/16, W-cycle, 4-CTA clusters, the host-buffer pipeline)."""
 import sys
 import numpy as np, torch
 sys.path.insert(0, '.')
@@ -12,9 +11,9 @@ kw = {}
 if mode == "wcycle":
     mats = [mats[4], mats[6]]
     kw = dict(force_path=wc.PATH_WCYCLE)
-if mode == "split":  # two warps per column-block pair (w = 16 shapes)
-    mats = [mats[4], workloads.gaussian(workloads.matrix_rng(778, 0), 120, 160)]
-    kw = dict(pair_warps=2)
+if mode == "cluster":  # Gram-path matrices over 4-CTA clusters (w = 8 and 16 shapes)
+    mats = [mats[4], workloads.gaussian(workloads.matrix_rng(778, 0), 120, 160), mats[6]]
+    kw = dict(cluster_ctas=4)
 if mode == "host":  # wcsvd_batched_host: chunked copy / compute pipeline, uniform and mixed
     A = torch.from_numpy(np.stack([workloads.gaussian(workloads.matrix_rng(779, i), 64, 64) for i in range(40)]))
     S, U, V, info = wc.svd_batched_host(A.pin_memory(), return_info=True)
