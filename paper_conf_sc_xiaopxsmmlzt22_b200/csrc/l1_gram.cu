@@ -160,25 +160,32 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-// Issue the copy of rows [r0, r0+16) of the 2w panel columns (offsets col_off[c] = pcol(c) * ld) into
-// ring stage `st`: W2 x 8 chunks of 16 B, W2/4 per lane.
+// Chunk addressing of a pair panel (2w columns = block I's w columns, then block J's): lane's chunk i
+// (W2/4 chunks of 16 B per lane and slab) is column c = lane/8 + 4i, i.e. block I for i < W2/8, block J
+// after, so two element offsets and 4 ld describe every chunk (instead of W2/4 registers).
+struct PanelAddr {
+  int aI, aJ;  // element offsets of this lane's first chunk column in block I / block J (+ row 2h)
+  int ld4;     // 4 ld
+};
 template <int W2>
-__device__ __forceinline__ void slab_issue(double* ring, const double* base, const int (&coff)[W2 / 4], int r0,
-                                           int st, int lane) {
-  constexpr int SL = WarpSmem<W2>::SL;
-  double* dst = ring + st * WarpSmem<W2>::SLAB;
-#pragma unroll
-  for (int i = 0; i < W2 / 4; ++i) {
-    const int q = lane + 32 * i, c = q >> 3, h = q & 7;
-    cp_async16(dst + c * SL + 2 * h, base + coff[i] + r0 + 2 * h);
-  }
+__device__ __forceinline__ PanelAddr panel_addr(int I, int J, int ld, int lane) {
+  constexpr int W = W2 / 2;
+  const int c0 = lane >> 3, h = lane & 7;
+  return PanelAddr{(I * W + c0) * ld + 2 * h, (J * W + c0) * ld + 2 * h, 4 * ld};
 }
 
-// Column offsets (pcol(c) * ld) of the chunks this lane copies.
+// Issue the copy of rows [r0, r0+16) of the 2w panel columns into ring stage `st`: W2 x 8 chunks of
+// 16 B, W2/4 per lane.
 template <int W2>
-__device__ __forceinline__ void slab_offsets(int (&coff)[W2 / 4], int I, int J, int ld, int lane) {
+__device__ __forceinline__ void slab_issue(double* ring, const double* base, const PanelAddr& pa, int r0, int st,
+                                           int lane) {
+  constexpr int SL = WarpSmem<W2>::SL, HI = W2 / 8;
+  double* dst = ring + st * WarpSmem<W2>::SLAB + (lane >> 3) * SL + 2 * (lane & 7);
 #pragma unroll
-  for (int i = 0; i < W2 / 4; ++i) coff[i] = pcol<W2>((lane + 32 * i) >> 3, I, J) * ld;
+  for (int i = 0; i < W2 / 4; ++i) {
+    const int off = (i < HI ? pa.aI + i * pa.ld4 : pa.aJ + (i - HI) * pa.ld4) + r0;
+    cp_async16(dst + 4 * i * SL, base + off);
+  }
 }
 
 // Upper tiles of P^T P for the global panel of pair (I, J): slabs stream through the NS-stage ring
@@ -189,17 +196,16 @@ __device__ __forceinline__ void gram_tiles_async(double* ring, const double* bas
   constexpr int CG = W2 / 8, SL = WarpSmem<W2>::SL;
 #pragma unroll
   for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
-  int coff[W2 / 4];
-  slab_offsets<W2>(coff, I, J, ld, lane);
+  const PanelAddr pa = panel_addr<W2>(I, J, ld, lane);
   const int nslab = rows >> 4;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ring, base, coff, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2>(ring, base, pa, 16 * j, j, lane);
     cp_async_commit();
   }
   const int fo = (lane >> 2) * SL + (lane & 3);  // fragment offset inside a column group
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
@@ -220,22 +226,19 @@ template <int W2, int NS>
 __device__ __forceinline__ void apply_rotation_async(double* ring, double* base, int ld, int rows, int I, int J,
                                                      int lane, const double (&jf)[W2 / 4][W2 / 8]) {
   constexpr int CG = W2 / 8, KK = W2 / 4, SL = WarpSmem<W2>::SL;
-  int coff[W2 / 4];
-  slab_offsets<W2>(coff, I, J, ld, lane);
-  int oc[CG][2];
-#pragma unroll
-  for (int nb = 0; nb < CG; ++nb)
-#pragma unroll
-    for (int e = 0; e < 2; ++e) oc[nb][e] = pcol<W2>(8 * nb + 2 * (lane & 3) + e, I, J) * ld + (lane >> 2);
+  const PanelAddr pa = panel_addr<W2>(I, J, ld, lane);
+  // output element offsets: column 8 nb + 2 (lane % 4) + e of the panel, row lane / 4 (+ 8h, + 16 sl)
+  constexpr int W = W2 / 2, HB = CG / 2;
+  const int oI = (I * W + 2 * (lane & 3)) * ld + (lane >> 2), oJ = (J * W + 2 * (lane & 3)) * ld + (lane >> 2);
   const int nslab = rows >> 4;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ring, base, coff, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2>(ring, base, pa, 16 * j, j, lane);
     cp_async_commit();
   }
   const int fo = (lane & 3) * SL + (lane >> 2);  // A fragment: row l/4, column l%4
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, coff, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
@@ -255,7 +258,9 @@ __device__ __forceinline__ void apply_rotation_async(double* ring, double* base,
 #pragma unroll
       for (int nb = 0; nb < CG; ++nb)
 #pragma unroll
-        for (int e = 0; e < 2; ++e) __stcg(base + oc[nb][e] + 16 * sl + 8 * h, acc[nb][e]);
+        for (int e = 0; e < 2; ++e)
+          __stcg(base + (nb < HB ? oI + (8 * nb + e) * ld : oJ + (8 * (nb - HB) + e) * ld) + 16 * sl + 8 * h,
+                 acc[nb][e]);
     }
     __syncwarp();
   }
@@ -1059,7 +1064,11 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
       if (crank == 0 && tid == 0) s_flags[sweep & 1] = 0;
       if (!any) { converged = true; break; }
     }
+#ifdef WCSVD_EXP_FLAT_WITH_WCYCLE
+  } else if ((MODE == kWcycle || (MODE == kFlat && d.w2 != 0)) && !nonfinite) {
+#else
   } else if (MODE == kWcycle && !nonfinite) {
+#endif
     // W-cycle (Alg 2 l.12-14; Step 3; Fig 3-4): Level-1 super-blocks
     // of width w1 = d.w are paired round-robin; each super-pair panel [A_I A_J] (M x 2 w1) fits no
     // on-chip EVD, so it recurses to Level 2: block Jacobi with w2 = d.w2 (the EVD width W2/2) over
