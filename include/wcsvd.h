@@ -63,7 +63,9 @@ enum {
   WCSVD_PATH_AUTO = 0,
   WCSVD_PATH_L0 = 1,      /* whole matrix on-chip: vector-rotation Jacobi, Alg 2 l.2-3 */
   WCSVD_PATH_GRAM = 2,    /* Level 1: Gram -> EVD(B_ij) -> GEMM update, Alg 2 l.10-11 */
-  WCSVD_PATH_WCYCLE = 3   /* Level 1 -> Level 2 recursion on each pair panel, Alg 2 l.12-14 */
+  WCSVD_PATH_WCYCLE = 3,  /* Level 1 -> Level 2 recursion on each pair panel, Alg 2 l.12-14 */
+  WCSVD_PATH_PANEL = 4    /* Level 1, J from the SVD of the pair panel (group (i), Alg 2 l.8-9): one-sided
+                             Jacobi of its CholeskyQR factor R (2w x 2w) in registers; w = 16, fp64 */
 };
 
 /* wcsvd_batched -- batched economy SVD.

@@ -18,12 +18,12 @@ from typing import Sequence
 import numpy as np
 
 __all__ = ["svd_batched", "svd_batched_host", "etkf_analysis", "svd_batched_raw", "plan", "round_robin", "lib", "WcsvdError",
-           "PATH_L0", "PATH_GRAM", "PATH_WCYCLE", "L0_TWO_PHASE_VARIANTS", "library_path"]
+           "PATH_L0", "PATH_GRAM", "PATH_WCYCLE", "PATH_PANEL", "L0_TWO_PHASE_VARIANTS", "library_path"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.environ.get("WCSVD_LIBRARY") or os.path.join(_HERE, "libwcsvd.so")  # env: experiment builds
 
-PATH_AUTO, PATH_L0, PATH_GRAM, PATH_WCYCLE = 0, 1, 2, 3
+PATH_AUTO, PATH_L0, PATH_GRAM, PATH_WCYCLE, PATH_PANEL = 0, 1, 2, 3, 4
 # Level-0 kernel variants that run the two-phase kernel (csrc/kernels.h kTP32, kTP64; csrc/l0_tp.cu)
 L0_TWO_PHASE_VARIANTS = (7, 8)
 WCSVD_OK, WCSVD_ENOTSUP, WCSVD_ECUDA, WCSVD_ENOMEM = 0, -100, -101, -102

@@ -14,6 +14,7 @@
 
 #include "common.cuh"
 #include "kernels.h"
+#include "plan_table.h"
 #include "wcsvd.h"
 
 namespace wcsvd {
@@ -50,6 +51,24 @@ int l0tp_variant(int M, int N) {
   return 0;
 }
 
+// Measured plan table (plan_table.h, tools/autotune.py + tools/gen_plan_table.py): the
+// entry nearest to (M, N) in (log N, log M/N), restricted to entries on the same side of the Level-0
+// fit (a matrix that fits one CTA is compared with measured shapes that also fit, and vice versa).
+const PlanEntry* plan_lookup(int M, int N, bool l0fit) {
+  const PlanEntry* best = nullptr;
+  double bd = 0;
+  const double ln = std::log((double)N), la = std::log((double)M / N);
+  for (int i = 0; i < kPlanTableSize; ++i) {
+    const PlanEntry& e = kPlanTable[i];
+    const int v = l0tp_variant(e.M, e.N) ? 1 : l0_variant(e.M, e.N);
+    if ((v != 0) != l0fit) continue;
+    const double dn = std::log((double)e.N) - ln, da = std::log((double)e.M / e.N) - la;
+    const double dd = dn * dn + da * da;
+    if (!best || dd < bd) { best = &e; bd = dd; }
+  }
+  return best;
+}
+
 int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   std::memset(p, 0, sizeof(*p));
   p->m = m;
@@ -60,8 +79,12 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   p->cost = f_tb(p->M, p->N);
   const int tp = l0tp_variant(p->M, p->N);
   const int v = tp ? tp : l0_variant(p->M, p->N);
-  // Alg 2 l.2: "if SVD of A^k can be implemented entirely within SM" -> Level 0.
-  if (v && (force_path == 0 || force_path == WCSVD_PATH_L0)) {
+  // Alg 2 l.2-14 level choice with the B200 measurements deciding among the
+  // paths that apply: Level 0 only if the matrix fits one CTA AND the nearest measured shape ran
+  // fastest on Level 0; the Gram-path EVD width and the W-cycle from the same table.
+  const PlanEntry* pe = (force_path == 0 && force_w == 0) ? plan_lookup(p->M, p->N, v != 0) : nullptr;
+  const bool take_l0 = v && (force_path == WCSVD_PATH_L0 || (force_path == 0 && (!pe || pe->path == WCSVD_PATH_L0)));
+  if (take_l0) {
     p->path = WCSVD_PATH_L0;
     p->variant = v;
     static const int np_of[] = {0, 8, 16, 32, 32, 48, 64, 32, 64};
@@ -71,10 +94,20 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   }
   if (force_path == WCSVD_PATH_L0) return WCSVD_ENOTSUP;
   // Alg 2 l.5-11: Level 1, column blocks of width w; the pair Gram's EVD runs on-chip.
-  int w = (p->N <= 96) ? 8 : 16;
+  int w = pe ? (pe->path == WCSVD_PATH_L0 ? pe->wg : pe->w) : ((p->N <= 96) ? 8 : 16);
   if (force_w == 8 || force_w == 16) w = force_w;
   else if (force_w != 0) return WCSVD_ENOTSUP;
-  if (force_path == WCSVD_PATH_WCYCLE) {
+  if (force_path == WCSVD_PATH_PANEL || (pe && pe->path == WCSVD_PATH_PANEL)) {
+    // Alg 2 l.8-9, group (i): J from the SVD of the pair panel (l1_gram.cu evd_fast32); w = 16
+    if (force_w == 8) return WCSVD_ENOTSUP;
+    p->path = WCSVD_PATH_PANEL;
+    p->w = 16;
+    p->n_pad = (p->N + 31) / 32 * 32;
+    p->m_pad = (p->M + 15) / 16 * 16;
+    p->variant = (p->n_pad / 32 >= 8) ? kL1_32x8 : kL1_32x4;
+    return WCSVD_OK;
+  }
+  if (force_path == WCSVD_PATH_WCYCLE || (pe && pe->path == WCSVD_PATH_WCYCLE)) {
     // Alg 2 l.12-14: w1 = 64 super-blocks recurse to Level 2 with w2 = w (EVD width 2 w2).
     p->path = WCSVD_PATH_WCYCLE;
     p->w = 64;
@@ -291,7 +324,7 @@ int validate(int batch, const int* m, const int* n, const TI* const* A, const in
     const int c = opts->cluster_ctas;
     if (c != 0 && c != 1 && c != 2 && c != 4 && c != 8) return -12;
     if (opts->f32_compute != 0 && opts->f32_compute != 1) return -12;
-    if (opts->force_path < 0 || opts->force_path > WCSVD_PATH_WCYCLE) return -12;
+    if (opts->force_path < 0 || opts->force_path > WCSVD_PATH_PANEL) return -12;
     if (opts->force_w != 0 && opts->force_w != 8 && opts->force_w != 16) return -12;
     for (int b = 0; b < batch; ++b) {
       wcsvd_plan_t p;
@@ -332,6 +365,7 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
   CallPlan cp;
   const int rc0 = make_call_plan(batch, m, n, force_path, force_w, opts ? opts->cluster_ctas : 0, &withv, &cp,
                                  tailor_total);
+  // (the fp32 FFMA route, opts->f32_compute = 1, has no PANEL variant: such buckets run fp64-inside)
   if (rc0 != WCSVD_OK) return rc0;
   const auto& plans = cp.plans;
   const auto& buckets = cp.buckets;
@@ -434,7 +468,8 @@ static int batched_impl(int batch, const int* m, const int* n, const TI* const* 
     else if (bk.path == WCSVD_PATH_L0)
       e = launch_l0(bk.variant, bk.withv, kF32 ? 1 : 0, d_descs, d_order + bucket_off[i], cnt, bk.maxM, st);
     else
-      e = launch_l1(bk.variant, bk.path == WCSVD_PATH_WCYCLE ? 1 : 0, kF32 ? 1 : 0, (opts && opts->f32_compute) ? 1 : 0,
+      e = launch_l1(bk.variant, bk.path == WCSVD_PATH_WCYCLE ? 1 : (bk.path == WCSVD_PATH_PANEL ? 2 : 0), kF32 ? 1 : 0,
+                    (opts && opts->f32_compute && bk.path != WCSVD_PATH_PANEL) ? 1 : 0,
                     d_descs, d_order + bucket_off[i], cnt, bk.cluster, pool, st);
     if (e == cudaSuccess && nbk > 1) e = cudaEventRecord(done[i], st);
   }

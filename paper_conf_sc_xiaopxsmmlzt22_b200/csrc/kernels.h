@@ -28,7 +28,8 @@ enum L1Variant {
 };
 
 // Level-1 launch: `cluster` CTAs per matrix (1, 2, 4 or 8; a thread-block cluster when > 1).
-// wcycle = 1: the W-cycle kernel (Level 1 -> Level 2 recursion, one CTA per matrix).
+// wcycle = 1: the W-cycle kernel (Level 1 -> Level 2 recursion, one CTA per matrix); 2: the group (i)
+// PANEL path (one-sided Jacobi of the CholeskyQR-compressed pair panel, 2w = 32, fp64 working copy).
 // fp32 = 1: float I/O; f32_compute = 1 iterates in fp32 (FFMA), else on an fp64 working copy (DMMA).
 cudaError_t launch_l1(int variant, int wcycle, int fp32, int f32_compute, const MatDesc* descs, const int* order,
                       int count, int cluster, const SlotPool& pool, cudaStream_t stream);

@@ -425,9 +425,137 @@ __device__ __forceinline__ bool evd_step(const T* __restrict__ Bc, T* __restrict
   return true;
 }
 
+// ---- Group (i) inner solve, PANEL path (Alg 2 l.8-9; Step 2 group (i), PAPER.md:175;
+// DESIGN.md §5.2c): J from the SVD of the pair panel P = [A_i A_j] itself, by one-sided Jacobi. The M x 2w
+// panel does not fit one warp's registers, so it is first compressed to its 2w x 2w triangular factor R
+// (P = Q R, Q orthonormal; R from the Cholesky factorisation of the Gram B = P^T P = R^T R -- CholeskyQR):
+// one-sided Jacobi on the columns of R produces exactly the rotations of one-sided Jacobi on the
+// columns of P (same alpha = ||p_i||^2, beta, gamma = p_i^T p_j), eq (3)-(4) PAPER.md:76-81. Cholesky:
+// lane c holds row / column c of B, pivots broadcast by shuffle, the trailing update reads row j of R
+// from a shared row buffer; R is then transposed so that lane r holds row r of R. Per step: 16 products, a
+// fixed-order butterfly reduce-scatter of the 16 dot products (lane L ends with pair L/2's gamma),
+// eq (4) in the pair's two lanes, eq (6) norm updates, the (c, s) of the step logged
+// to shared memory, and the 16 column rotations of the lane's row with register renaming. J is built
+// afterwards from the log. Falls back to the two-sided sweep when a Cholesky pivot falls below
+// 2^-24 of its column's norm^2 (nearly dependent columns: R would lose relative accuracy).
+constexpr double kCholTau = 5.9604644775390625e-08;  // 2^-24
+
+// One one-sided step: x = row `lane` of R (slot order) -> y (moved slots); alpha = ||column lane||^2.
+__device__ __forceinline__ bool onesided_step(const double (&x)[32], double (&y)[32], double& alpha,
+                                              double2* __restrict__ logs, int lane, double tol2) {
+  double v[16];
+#pragma unroll
+  for (int k = 0; k < 16; ++k) v[k] = x[2 * k] * x[2 * k + 1];
+  // butterfly reduce-scatter: level o keeps the half selected by lane bit log2(o), lane L -> pair L/2
+#pragma unroll
+  for (int o = 16, n = 8; o >= 2; o >>= 1, n >>= 1) {
+    const bool up = (lane & o) != 0;
+#pragma unroll
+    for (int i = 0; i < n; ++i) {
+      const double keep = up ? v[n + i] : v[i];
+      const double send = up ? v[i] : v[n + i];
+      v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+    }
+  }
+  const double g = v[0] + __shfl_xor_sync(0xffffffffu, v[0], 1);  // gamma_{lane/2}, bitwise equal in both lanes
+  const double ao = __shfl_xor_sync(0xffffffffu, alpha, 1);
+  const bool odd = lane & 1;
+  const double ap = odd ? ao : alpha, aq = odd ? alpha : ao;  // (alpha_2k, alpha_2k+1) in both lanes
+  double c, s, t;
+  const bool rot = jacobi_rotation(ap, aq, g, tol2, c, s, t);
+  if (rot) alpha = odd ? fma(-t, g, alpha) : fma(t, g, alpha);  // eq (6)
+  if (!odd) logs[lane >> 1] = make_double2(c, s);
+  alpha = __shfl_sync(0xffffffffu, alpha, rr_src(lane, 32));  // norms move with their columns
+  const bool any = __any_sync(0xffffffffu, rot);
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < 16; ++k) {
+    const double2 q = logs[k];
+    const double a = x[2 * k], b = x[2 * k + 1];
+    y[rr_dest(2 * k, 32)] = fma(q.y, b, q.x * a);
+    y[rr_dest(2 * k + 1, 32)] = fma(-q.y, a, q.x * b);
+  }
+  return any;
+}
+
+// J <- J G of logged step `st` (or the rename only when the step did not rotate).
+__device__ __forceinline__ void jbuild_step(const double (&x)[32], double (&y)[32], const double2* logs, bool any) {
+  if (!any) {
+#pragma unroll
+    for (int k = 0; k < 32; ++k) y[rr_dest(k, 32)] = x[k];
+    return;
+  }
+#pragma unroll
+  for (int k = 0; k < 16; ++k) {
+    const double2 q = logs[k];
+    const double a = x[2 * k], b = x[2 * k + 1];
+    y[rr_dest(2 * k, 32)] = fma(q.y, b, q.x * a);
+    y[rr_dest(2 * k + 1, 32)] = fma(-q.y, a, q.x * b);
+  }
+}
+
+// Returns false (nothing changed) if the Cholesky route does not apply; else ja = J (row `lane`,
+// slot = original order) and *rotated.
+__device__ __forceinline__ bool evd_fast32(const double* __restrict__ B0, double* __restrict__ scratch, int lane,
+                                        double tol2, double (&ja)[32], bool* rotated) {
+  // scratch: >= 1056 doubles (transpose 32 x 33; the Cholesky row buffers and the (c, s) log alias it)
+  double b[32], r[32];
+#pragma unroll
+  for (int c = 0; c < 32; ++c) b[c] = B0[evd_phys_sym<32>(lane, c)];
+  const double dl = B0[evd_phys<32>(lane, lane)];  // ||column lane||^2 (original)
+  bool ok = true;
+#pragma unroll
+  for (int j = 0; j < 32; ++j) {
+    const double d = __shfl_sync(0xffffffffu, b[j], j);
+    const double d0 = __shfl_sync(0xffffffffu, dl, j);
+    ok &= !(d0 > 0.0) || d > kCholTau * d0;
+    const double inv = (d0 > 0.0 && d > 0.0) ? rsqrt(d) : 0.0;
+    const double rj = (lane >= j) ? b[j] * inv : 0.0;  // R[j][lane]
+    r[j] = rj;
+    double* rb = scratch + 32 * (j & 1);
+    rb[lane] = rj;
+    __syncwarp();
+#pragma unroll
+    for (int c = j + 1; c < 32; ++c) b[c] = fma(-rj, rb[c], b[c]);
+  }
+  if (!ok) return false;  // warp-uniform (every lane saw every pivot)
+  __syncwarp();
+  // transpose: lane c holds column c of R (r[j] = R[j][c]); lane r needs row r
+#pragma unroll
+  for (int j = 0; j < 32; ++j) scratch[j * 33 + lane] = r[j];
+  __syncwarp();
+#pragma unroll
+  for (int c = 0; c < 32; ++c) b[c] = scratch[lane * 33 + c];
+  __syncwarp();
+  double alpha = dl;
+  double2* logs = reinterpret_cast<double2*>(scratch);  // [31][16]
+  unsigned mask = 0;
+  // 31 steps (odd): x->y first, then pairs y->x, x->y; slots return to the original order
+  mask |= (unsigned)onesided_step(b, r, alpha, logs, lane, tol2);
+#pragma unroll 1
+  for (int st = 1; st < 31; st += 2) {
+    mask |= (unsigned)onesided_step(r, b, alpha, logs + 16 * st, lane, tol2) << st;
+    mask |= (unsigned)onesided_step(b, r, alpha, logs + 16 * (st + 1), lane, tol2) << (st + 1);
+  }
+  *rotated = mask != 0;
+  if (!mask) return true;
+  // J = product of the logged step rotations (slot order, rows in lanes)
+#pragma unroll
+  for (int s = 0; s < 32; ++s) b[s] = (lane == s) ? 1.0 : 0.0;
+  jbuild_step(b, r, logs, mask & 1u);
+#pragma unroll 1
+  for (int st = 1; st < 31; st += 2) {
+    jbuild_step(r, b, logs + 16 * st, (mask >> st) & 1u);
+    jbuild_step(b, r, logs + 16 * (st + 1), (mask >> (st + 1)) & 1u);
+  }
+#pragma unroll
+  for (int s = 0; s < 32; ++s) ja[s] = r[s];
+  return true;
+}
+
 // Process one column-block pair (I, J) of the working matrix with one warp. Returns true if it
 // rotated (A and V panels updated); counts inner sweeps into *inner.
-template <int W2>
+template <int W2, bool PANEL = false>
 __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, double* Wm, int ld, int mrows,
                              double* Vm, int ldv, int vrows, int I, int J, double tol2, int inner_cap,
                              int lane, int* inner) {
@@ -472,7 +600,13 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   double ja[W2], jb[W2];
   bool rotated = false;
   int isw = 0;
-  {
+  bool panel_done = false;
+  if constexpr (PANEL && W2 == 32) {
+    // group (i): one-sided Jacobi of the (CholeskyQR-compressed) panel; group (ii) below if a pivot is tiny
+    if (inner_cap == 1) panel_done = evd_fast32(B0, B1, lane, tol2, ja, &rotated);
+    if (panel_done) isw = 1;
+  }
+  if (!panel_done) {
   EvdMap<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
   em.init(lane);
 #pragma unroll
@@ -853,7 +987,7 @@ __host__ __device__ constexpr size_t warp_stride() {
 // MODE: kFlat (flat Gram path, one CTA per matrix), kFlatCluster (flat Gram path, a cluster of CTAs
 // per matrix), kWcycle (Level 1 -> Level 2 recursion, one CTA). Separate instantiations keep one
 // inlined copy of process_pair per kernel (register pressure).
-enum { kFlat = 0, kFlatCluster = 1, kWcycle = 2 };
+enum { kFlat = 0, kFlatCluster = 1, kWcycle = 2, kPanel = 3 };
 
 template <int W2, int NW, typename TI, typename TW, int MODE>
 __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
@@ -1047,7 +1181,8 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
           if constexpr (F32)
             rot_any |= process_pair_f32<W2>(wsf, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
           else
-            rot_any |= process_pair<W2>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap, lane, &my_inner);
+            rot_any |= process_pair<W2, MODE == kPanel>(ws, s_em, Wm, mp, mp, Vm, np, vrows, I, J, tol2, d.inner_cap,
+                                                        lane, &my_inner);
           pair_fence<CLU>();  // every lane's W / V writes precede ...
           __syncwarp();
           if (lane == 0) {    // ... the release
@@ -1252,6 +1387,10 @@ static cudaError_t launch_l1_t(const MatDesc* descs, const int* order, int count
 template <typename TI, typename TW, int W2, int NW>
 static cudaError_t launch_l1_m(int wcycle, const MatDesc* descs, const int* order, int count, int cluster,
                                const SlotPool& pool, cudaStream_t stream) {
+  if (wcycle == 2) {  // group (i) PANEL path: fp64, 2w = 32
+    if constexpr (W2 == 32 && sizeof(TW) == 8) return launch_l1_t<W2, NW, TI, TW, kPanel>(descs, order, count, 1, pool, stream);
+    return cudaErrorInvalidValue;
+  }
   if (wcycle) return launch_l1_t<W2, NW, TI, TW, kWcycle>(descs, order, count, 1, pool, stream);
   if (cluster > 1) return launch_l1_t<W2, NW, TI, TW, kFlatCluster>(descs, order, count, cluster, pool, stream);
   return launch_l1_t<W2, NW, TI, TW, kFlat>(descs, order, count, 1, pool, stream);

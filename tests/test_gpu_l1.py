@@ -119,3 +119,29 @@ def test_removed_split_executor_is_rejected():
     with pytest.raises(wcm.WcsvdError) as ei:
         wcm.svd_batched(A, pair_warps=2)
     assert ei.value.code == -12
+
+
+@pytest.mark.parametrize("shapes", [
+    [(256, 256), (300, 170), (170, 300), (1024, 128), (97, 97), (513, 257)],
+    [(64, 64), (40, 33), (33, 65)],
+])
+def test_panel_path_group_i(shapes):
+    # group (i) (Alg 2 l.8-9): J from one-sided Jacobi of the CholeskyQR-compressed pair panel
+    mats = [workloads.gaussian(workloads.matrix_rng(590 + i, 9), m, n) for i, (m, n) in enumerate(shapes)]
+    for (m, n) in shapes:
+        assert wc.plan(m, n, force_path=wc.PATH_PANEL)["path"] == wc.PATH_PANEL
+    S, U, V, info = gpu_svd_list(mats, force_path=wc.PATH_PANEL)
+    check_parity(mats, S, U, V, info)
+
+
+def test_panel_path_ill_conditioned_falls_back_per_pair():
+    # nearly dependent / rank-deficient panels take the two-sided EVD for that pair (tiny Cholesky pivot)
+    rng = workloads.matrix_rng(595, 0)
+    s = 1e12 ** (-np.arange(150) / 149.0)
+    A1 = workloads.prescribed(rng, 200, 150, s)
+    Z = workloads.gaussian(rng, 180, 130)
+    Z[:, 5] = 0.0
+    Z[:, 77] = Z[:, 3]
+    mats = [A1, Z]
+    S, U, V, info = gpu_svd_list(mats, force_path=wc.PATH_PANEL)
+    check_parity(mats, S, U, V, info)
