@@ -34,6 +34,11 @@
 #ifndef WCSVD_L1_NS
 #define WCSVD_L1_NS 1
 #endif
+// fp64 inner EVD storage: 1 = full symmetric B, select-free quads (evd_step_full), 0 = upper triangle in
+// the swizzled slot layout (evd_step; round-1 kernel, A/B builds)
+#ifndef WCSVD_EVD_FULL
+#define WCSVD_EVD_FULL 1
+#endif
 #ifndef WCSVD_L1_NSTAGE
 #define WCSVD_L1_NSTAGE 3
 #endif
@@ -425,6 +430,108 @@ __device__ __forceinline__ bool evd_step(const T* __restrict__ Bc, T* __restrict
   return true;
 }
 
+// ---- Inner EVD step, full-symmetric layout (default, WCSVD_EVD_FULL = 1) ----
+// B is stored as the FULL symmetric 2w x 2w matrix in slot order (row stride 2w, both triangles). Lane
+// L works for pair k = L mod w (its own rotation) and owns the quads B(k, l), l = k + d (mod w), for its
+// share of d: with both triangles stored, the quad is always loaded as rows (2k, 2k+1) x columns
+// (2l, 2l+1) -- lane-uniform shape, no swaps and no "which side am I" selects -- rotated by the lane's
+// own (c, s) on the rows and the partner's (c, s) (one shuffle from lane l) on the columns, and written
+// with its transpose to the slots both index pairs move to. A quarter-warp's eight LDS.128 hit eight
+// distinct 16-byte bank groups (group = (k + d) mod 8), so no swizzle is needed.
+template <int W2>
+struct EvdMapF {
+  static constexpr int NPR = W2 / 2, LPP = 32 / NPR, HALF = NPR / 2;
+  static constexpr int QPL = (HALF + LPP - 1) / LPP;
+  int ld[QPL];      // bits 0-11 load offset of B(2k, 2l); bits 12-16 partner l; bit 17 valid
+  int st[QPL][4];   // store offsets (16-bit pairs) of the quad and of its transpose
+  int dld, dst[2];  // diagonal block load offset (2k, 2k); stores (moved slots): (p,p) | (q,q) << 16, (p,q) | (q,p) << 16
+  __device__ __forceinline__ void init(int lane) {
+    const int k = lane & (NPR - 1), h = lane / NPR;
+    const int k0 = rr_dest(2 * k, W2), k1 = rr_dest(2 * k + 1, W2);
+#pragma unroll
+    for (int i = 0; i < QPL; ++i) {
+      const int d = 1 + h * QPL + i;
+      const bool valid = d < HALF || (d == HALF && k < HALF);
+      const int l = (k + d) & (NPR - 1);
+      const int l0 = rr_dest(2 * l, W2), l1 = rr_dest(2 * l + 1, W2);
+      ld[i] = valid ? ((2 * k) * W2 + 2 * l) | (l << 12) | (1 << 17) : 0;
+      st[i][0] = (k0 * W2 + l0) | ((k0 * W2 + l1) << 16);
+      st[i][1] = (k1 * W2 + l0) | ((k1 * W2 + l1) << 16);
+      st[i][2] = (l0 * W2 + k0) | ((l1 * W2 + k0) << 16);  // transpose: B'(l, k) = B'(k, l)^T
+      st[i][3] = (l0 * W2 + k1) | ((l1 * W2 + k1) << 16);
+    }
+    dld = (2 * k) * W2 + 2 * k;
+    dst[0] = (k0 * W2 + k0) | ((k1 * W2 + k1) << 16);
+    dst[1] = (k0 * W2 + k1) | ((k1 * W2 + k0) << 16);
+  }
+};
+
+template <int W2>
+__device__ __forceinline__ bool evd_step_full(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
+                                              const EvdMapF<W2>& em, int lane, double tol2, const double (&x)[W2],
+                                              double (&y)[W2]) {
+  constexpr int NPR = W2 / 2, QPL = EvdMapF<W2>::QPL;
+  const double2 dv0 = *reinterpret_cast<const double2*>(Bc + em.dld);       // b_pp, b_pq
+  const double bqq = Bc[em.dld + W2 + 1];
+  double c, s, t;
+  const bool rot = jacobi_rotation(dv0.x, bqq, dv0.y, tol2, c, s, t);
+  double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
+#pragma unroll
+  for (int i = 0; i < QPL; ++i) {
+    if (em.ld[i] & (1 << 17)) {
+      const int o = em.ld[i] & 0xfff;
+      const double2 v0 = *reinterpret_cast<const double2*>(Bc + o);
+      const double2 v1 = *reinterpret_cast<const double2*>(Bc + o + W2);
+      b00[i] = v0.x; b01[i] = v0.y; b10[i] = v1.x; b11[i] = v1.y;
+    }
+  }
+  if (lane < NPR) {
+    cs[lane] = make_double2(c, s);
+    const double pp = rot ? fma(t, dv0.y, dv0.x) : dv0.x, qq = rot ? fma(-t, dv0.y, bqq) : bqq;
+    const double pq = rot ? 0.0 : dv0.y;
+    Bn[em.dst[0] & 0xffff] = pp;
+    Bn[em.dst[0] >> 16] = qq;
+    Bn[em.dst[1] & 0xffff] = pq;
+    Bn[em.dst[1] >> 16] = pq;
+  }
+  const bool any = __any_sync(0xffffffffu, rot);
+#pragma unroll
+  for (int i = 0; i < QPL; ++i) {
+    const int l = (em.ld[i] >> 12) & 31;
+    const double cl = __shfl_sync(0xffffffffu, c, l), sl = __shfl_sync(0xffffffffu, s, l);
+    if (em.ld[i] & (1 << 17)) {
+      // columns (2l, 2l+1): B G_l; rows (2k, 2k+1): G_k^T (B G_l)
+      const double c0 = fma(sl, b01[i], cl * b00[i]), c1 = fma(-sl, b00[i], cl * b01[i]);
+      const double d0 = fma(sl, b11[i], cl * b10[i]), d1 = fma(-sl, b10[i], cl * b11[i]);
+      const double n00 = fma(s, d0, c * c0), n01 = fma(s, d1, c * c1);
+      const double n10 = fma(-s, c0, c * d0), n11 = fma(-s, c1, c * d1);
+      Bn[em.st[i][0] & 0xffff] = n00;
+      Bn[em.st[i][0] >> 16] = n01;
+      Bn[em.st[i][1] & 0xffff] = n10;
+      Bn[em.st[i][1] >> 16] = n11;
+      Bn[em.st[i][2] & 0xffff] = n00;  // (l0, k0)
+      Bn[em.st[i][2] >> 16] = n01;     // (l1, k0)
+      Bn[em.st[i][3] & 0xffff] = n10;  // (l0, k1)
+      Bn[em.st[i][3] >> 16] = n11;     // (l1, k1)
+    }
+  }
+  if (!any) {
+#pragma unroll
+    for (int k = 0; k < W2; ++k) y[rr_dest(k, W2)] = x[k];
+    return false;
+  }
+  __syncwarp();
+  // J <- J G in slot order; outputs move to their next slots (register rename).
+#pragma unroll
+  for (int k = 0; k < NPR; ++k) {
+    const double2 g = cs[k];
+    const double a = x[2 * k], b = x[2 * k + 1];
+    y[rr_dest(2 * k, W2)] = fma(g.y, b, g.x * a);
+    y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
+  }
+  return true;
+}
+
 // ---- Group (i) inner solve, PANEL path (Alg 2 l.8-9; Step 2 group (i), PAPER.md:175;
 // DESIGN.md §5.2c): J from the SVD of the pair panel P = [A_i A_j] itself, by one-sided Jacobi. The M x 2w
 // panel does not fit one warp's registers, so it is first compressed to its 2w x 2w triangular factor R
@@ -501,8 +608,13 @@ __device__ __forceinline__ bool evd_fast32(const double* __restrict__ B0, double
   // scratch: >= 1056 doubles (transpose 32 x 33; the Cholesky row buffers and the (c, s) log alias it)
   double b[32], r[32];
 #pragma unroll
+#if WCSVD_EVD_FULL
+  for (int c = 0; c < 32; ++c) b[c] = B0[lane * 32 + c];
+  const double dl = B0[lane * 33];  // ||column lane||^2 (original)
+#else
   for (int c = 0; c < 32; ++c) b[c] = B0[evd_phys_sym<32>(lane, c)];
-  const double dl = B0[evd_phys<32>(lane, lane)];  // ||column lane||^2 (original)
+  const double dl = B0[evd_phys<32>(lane, lane)];
+#endif
   bool ok = true;
 #pragma unroll
   for (int j = 0; j < 32; ++j) {
@@ -576,7 +688,12 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
 #pragma unroll
         for (int e = 0; e < 2; ++e) {
           const int row = 8 * a + (lane >> 2), col = 8 * b + 2 * (lane & 3) + e;
+#if WCSVD_EVD_FULL
+          B0[row * W2 + col] = acc[t][e];
+          if (a != b) B0[col * W2 + row] = acc[t][e];
+#else
           if (a != b || row <= col) B0[evd_phys<W2>(row, col)] = acc[t][e];
+#endif
         }
   }
   __syncwarp();
@@ -584,11 +701,17 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   // (4) off-norm test on the Gram (Z6): skip the pair if every b_pq^2 <= tol^2 b_pp b_qq.
   bool need = false;
   {
-    const double bqq = (lane < W2) ? B0[evd_phys<W2>(lane, lane)] : 0.0;
+#if WCSVD_EVD_FULL
+#define BIDX(a, b) ((a) * W2 + (b))
+#else
+#define BIDX(a, b) evd_phys<W2>(a, b)
+#endif
+    const double bqq = (lane < W2) ? B0[BIDX(lane, lane)] : 0.0;
 #pragma unroll 4
     for (int p = 0; p < W2 - 1; ++p) {
-      const double bpp = B0[evd_phys<W2>(p, p)];  // broadcast
-      const double bpq = (lane < W2 && lane > p) ? B0[evd_phys<W2>(p, lane)] : 0.0;
+      const double bpp = B0[BIDX(p, p)];  // broadcast
+      const double bpq = (lane < W2 && lane > p) ? B0[BIDX(p, lane)] : 0.0;
+#undef BIDX
       const double ab = bpp * bqq;
       need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
     }
@@ -607,20 +730,27 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
     if (panel_done) isw = 1;
   }
   if (!panel_done) {
-  EvdMap<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
+#if WCSVD_EVD_FULL
+  EvdMapF<W2> em;  // lane-static map, rebuilt per pair (no registers held outside the EVD)
+#define EVD_STEP evd_step_full<W2>
+#else
+  EvdMap<W2> em;
+#define EVD_STEP evd_step<W2>
+#endif
   em.init(lane);
 #pragma unroll
   for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
   for (; isw < inner_cap; ++isw) {
     // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb / B1, slots back in order.
-    bool any = evd_step<W2>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+    bool any = EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja, jb);
     __syncwarp();
     for (int r = 1; r < W2 - 1; r += 2) {
-      any |= evd_step<W2>(B1, B0, ws.cs, em, lane, tol2, jb, ja);
+      any |= EVD_STEP(B1, B0, ws.cs, em, lane, tol2, jb, ja);
       __syncwarp();
-      any |= evd_step<W2>(B0, B1, ws.cs, em, lane, tol2, ja, jb);
+      any |= EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja, jb);
       __syncwarp();
     }
+#undef EVD_STEP
 #pragma unroll
     for (int s = 0; s < W2; ++s) ja[s] = jb[s];
     double* tmp = B0;
