@@ -133,6 +133,12 @@ int plan_one(int m, int n, int force_path, int force_w, wcsvd_plan_t* p) {
   p->m_pad = (p->M + 15) / 16 * 16;
   const int pairs = p->n_pad / w / 2;
   p->variant = (w == 8) ? kL1_16x4 : (pairs >= 8 ? kL1_32x8 : kL1_32x4);
+  static const int env_nw = [] {  // experiments only: WCSVD_L1_NW=4 / 8 forces the 2w = 32 CTA width
+    const char* e = std::getenv("WCSVD_L1_NW");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (w == 16 && env_nw == 4) p->variant = kL1_32x4;
+  if (w == 16 && env_nw == 8) p->variant = kL1_32x8;
   return WCSVD_OK;
 }
 
@@ -148,7 +154,18 @@ size_t slot_doubles(const wcsvd_plan_t& p) {
 // l1_gram.cu launch bounds): the tailoring rule and the slot-pool capacity use them.
 int l1_warps(int variant) { return variant == kL1_32x8 ? 8 : 4; }
 int resident_per_sm(const wcsvd_plan_t& p) {
-  if (p.path == WCSVD_PATH_L0) return 4;  // two-phase kernels: 128 registers, <= 4 CTAs per SM
+  if (p.path == WCSVD_PATH_L0) {
+    // two-phase kernels: the slot pool must cover every CTA that can be resident (fp64 or fp32 build)
+    const int a = l0tp_occupancy(p.variant, 0, p.M), b = l0tp_occupancy(p.variant, 1, p.M);
+    const int r = a > b ? a : b;
+    if (r <= 0) cudaGetLastError();  // no device (CPU-side planning): clear the query's error
+    return r > 0 ? r : 8;
+  }
+  static const int env_res4 = [] {  // experiments only: builds with WCSVD_L1_MINB(4) = 3
+    const char* e = std::getenv("WCSVD_L1_RES4");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (p.variant == kL1_32x4 && env_res4 > 0) return env_res4;
   return p.variant == kL1_32x8 ? 1 : 2;
 }
 

@@ -37,6 +37,7 @@ cudaError_t launch_l1(int variant, int wcycle, int fp32, int f32_compute, const 
 cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
                         const SlotPool& pool, cudaStream_t stream);
 size_t l0tp_park_bytes(int variant, int M);  // per-matrix park buffer (X and V_x registers), fp64
+int l0tp_occupancy(int variant, int fp32, int maxM);  // resident CTAs per SM (-1 if unknown)
 
 cudaError_t launch_l0(int variant, int withv, int fp32, const MatDesc* descs, const int* order, int count,
                       int maxM, cudaStream_t stream);

@@ -43,6 +43,10 @@
 #ifndef WCSVD_EVD_ROT32
 #define WCSVD_EVD_ROT32 0
 #endif
+// Resident CTAs per SM the Level-1 kernels are compiled for (register budget 65536 / (32 NW minB)).
+#ifndef WCSVD_L1_MINB
+#define WCSVD_L1_MINB(nw) 1
+#endif
 #ifndef WCSVD_L1_NSTAGE
 #define WCSVD_L1_NSTAGE 3
 #endif
@@ -472,8 +476,7 @@ struct EvdMapF {
 
 template <int W2>
 __device__ __forceinline__ bool evd_step_full(const double* __restrict__ Bc, double* __restrict__ Bn, double2* cs,
-                                              const EvdMapF<W2>& em, int lane, double tol2, const double (&x)[W2],
-                                              double (&y)[W2]) {
+                                              const EvdMapF<W2>& em, int lane, double tol2, double (&x)[W2]) {
   constexpr int NPR = W2 / 2, QPL = EvdMapF<W2>::QPL;
   const double2 dv0 = *reinterpret_cast<const double2*>(Bc + em.dld);       // b_pp, b_pq
   const double bqq = Bc[em.dld + W2 + 1];
@@ -532,21 +535,28 @@ __device__ __forceinline__ bool evd_step_full(const double* __restrict__ Bc, dou
       Bn[em.st[i][3] >> 16] = n11;     // (l1, k1)
     }
   }
-  if (!any) {
+  if (any) __syncwarp();
+  // J <- J G in slot order, IN PLACE: every output goes straight into the register of the slot it
+  // moves to (common.cuh ring). Pairs are visited from the last to the first: the top output of
+  // pair k lands in top[k+1] (pair k+1 was already read), the bottom output is held one pair
+  // (`pend`) until pair k-1 has read bot[k-1]. One register set instead of the x -> y ping-pong
+  // (-64 registers); the same operations on the same operands, so the bits are unchanged.
+  double pend = 0.0;
 #pragma unroll
-    for (int k = 0; k < W2; ++k) y[rr_dest(k, W2)] = x[k];
-    return false;
-  }
-  __syncwarp();
-  // J <- J G in slot order; outputs move to their next slots (register rename).
-#pragma unroll
-  for (int k = 0; k < NPR; ++k) {
-    const double2 g = cs[k];
+  for (int k = NPR - 1; k >= 0; --k) {
     const double a = x[2 * k], b = x[2 * k + 1];
-    y[rr_dest(2 * k, W2)] = fma(g.y, b, g.x * a);
-    y[rr_dest(2 * k + 1, W2)] = fma(-g.y, a, g.x * b);
+    if (k < NPR - 1) x[2 * k + 1] = pend;
+    double na = a, nb = b;
+    if (any) {
+      const double2 g = cs[k];
+      na = fma(g.y, b, g.x * a);
+      nb = fma(-g.y, a, g.x * b);
+    }
+    x[rr_dest(2 * k, W2)] = na;
+    if (k >= 1) pend = nb;
+    else x[rr_dest(1, W2)] = nb;
   }
-  return true;
+  return any;
 }
 
 // ---- Group (i) inner solve, PANEL path (Alg 2 l.8-9; Step 2 group (i), PAPER.md:175;
@@ -758,6 +768,18 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
 #pragma unroll
   for (int s = 0; s < W2; ++s) ja[s] = (lane == s) ? 1.0 : 0.0;
   for (; isw < inner_cap; ++isw) {
+#if WCSVD_EVD_FULL
+    // W2-1 steps (odd): B ping-pongs B0 -> B1 -> B0 ..., ends in B1; J is updated in place in ja and
+    // its slots are back in order after the sweep.
+    bool any = EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja);
+    __syncwarp();
+    for (int r = 1; r < W2 - 1; r += 2) {
+      any |= EVD_STEP(B1, B0, ws.cs, em, lane, tol2, ja);
+      __syncwarp();
+      any |= EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja);
+      __syncwarp();
+    }
+#else
     // W2-1 steps (odd): x->y first, then pairs y->x, x->y; ends in jb / B1, slots back in order.
     bool any = EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja, jb);
     __syncwarp();
@@ -767,9 +789,10 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
       any |= EVD_STEP(B0, B1, ws.cs, em, lane, tol2, ja, jb);
       __syncwarp();
     }
-#undef EVD_STEP
 #pragma unroll
     for (int s = 0; s < W2; ++s) ja[s] = jb[s];
+#endif
+#undef EVD_STEP
     double* tmp = B0;
     B0 = B1;
     B1 = tmp;
@@ -1137,7 +1160,7 @@ __host__ __device__ constexpr size_t warp_stride() {
 enum { kFlat = 0, kFlatCluster = 1, kWcycle = 2, kPanel = 3 };
 
 template <int W2, int NW, typename TI, typename TW, int MODE>
-__global__ void __launch_bounds__(NW * 32, 1) l1_gram_kernel(const MatDesc* __restrict__ descs,
+__global__ void __launch_bounds__(NW * 32, WCSVD_L1_MINB(NW)) l1_gram_kernel(const MatDesc* __restrict__ descs,
                                                              const int* __restrict__ order, SlotPool pool) {
   // TI: type of A, S, U, V in the caller's memory (double, or float for wcsvd_batched_f32); the
   // iteration always runs on the fp64 working copy. CLU: the matrix is owned by a CTA cluster.
