@@ -173,6 +173,48 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+// L2 eviction priorities of the panel streams (WCSVD_L2HINT). The A panel a pair's Gram
+// reads is read again by the same pair's update one EVD later (short reuse); the V panel is touched
+// once per pair and next only one step later (long reuse). Hint kinds: 0 = the Gram's A loads, 1 = the
+// update's A loads / stores, 2 = the update's V loads / stores. Mode 0 = no hints (plain cp.async.cg /
+// st.global.cg). Measured (same box, ms, C3 / C4 / half of C5): none 226.1 / 339.0 / 1444; 1 (Gram A
+// evict_last, V evict_first) 219.6 / 340.7 / 1447; 2 (1 + update A loads evict_first) 222.2 / 340.6 /
+// 1452; 3 (2 + update A stores evict_last) 219.6 / 340.1 / 1446; 4 (V evict_first only) 219.6 / 339.7 /
+// 1450; C4 DRAM bytes unchanged (1.51 TB per launch) in every mode: at 2w = 32 the pair's working sets
+// in flight (8 per SM) exceed L2 whatever the priorities. Default 4: the V stream gives way.
+#ifndef WCSVD_L2HINT
+#define WCSVD_L2HINT 4
+#endif
+__device__ __forceinline__ unsigned long long l2_policy(int prio) {  // 0 evict_first, 1 normal, 2 evict_last
+  unsigned long long p;
+  if (prio == 0) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  else if (prio == 2) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  else asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// priority of loads (LD) or stores (ST) of hint kind K under WCSVD_L2HINT
+template <int K, bool ST>
+__device__ __forceinline__ constexpr int l2_prio() {
+#if WCSVD_L2HINT == 1
+  return K == 0 ? 2 : (K == 2 ? 0 : 1);
+#elif WCSVD_L2HINT == 2
+  return K == 0 ? 2 : (K == 2 ? 0 : (ST ? 1 : 0));
+#elif WCSVD_L2HINT == 3
+  return K == 0 ? 2 : (K == 2 ? 0 : (ST ? 2 : 0));
+#elif WCSVD_L2HINT == 4
+  return K == 2 ? 0 : 1;
+#else
+  return -1;
+#endif
+}
+__device__ __forceinline__ void cp_async16_hint(void* smem, const void* gmem, unsigned long long pol) {
+  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(sa), "l"(gmem), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st_hint(double* p, double v, unsigned long long pol) {
+  asm volatile("st.global.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(p), "d"(v), "l"(pol) : "memory");
+}
+
 // Chunk addressing of a pair panel (2w columns = block I's w columns, then block J's): lane's chunk i
 // (W2/4 chunks of 16 B per lane and slab) is column c = lane/8 + 4i, i.e. block I for i < W2/8, block J
 // after, so two element offsets and 4 ld describe every chunk (instead of W2/4 registers).
@@ -189,15 +231,16 @@ __device__ __forceinline__ PanelAddr panel_addr(int I, int J, int ld, int lane) 
 
 // Issue the copy of rows [r0, r0+16) of the 2w panel columns into ring stage `st`: W2 x 8 chunks of
 // 16 B, W2/4 per lane.
-template <int W2>
+template <int W2, int K = 1>
 __device__ __forceinline__ void slab_issue(double* ring, const double* base, const PanelAddr& pa, int r0, int st,
-                                           int lane) {
+                                           int lane, unsigned long long pol = 0ull) {
   constexpr int SL = WarpSmem<W2>::SL, HI = W2 / 8;
   double* dst = ring + st * WarpSmem<W2>::SLAB + (lane >> 3) * SL + 2 * (lane & 7);
 #pragma unroll
   for (int i = 0; i < W2 / 4; ++i) {
     const int off = (i < HI ? pa.aI + i * pa.ld4 : pa.aJ + (i - HI) * pa.ld4) + r0;
-    cp_async16(dst + 4 * i * SL, base + off);
+    if constexpr (l2_prio<K, false>() >= 0) cp_async16_hint(dst + 4 * i * SL, base + off, pol);
+    else cp_async16(dst + 4 * i * SL, base + off);
   }
 }
 
@@ -211,14 +254,15 @@ __device__ __forceinline__ void gram_tiles_async(double* ring, const double* bas
   for (int t = 0; t < PairCfg<W2>::NTU; ++t) acc[t][0] = acc[t][1] = 0.0;
   const PanelAddr pa = panel_addr<W2>(I, J, ld, lane);
   const int nslab = rows >> 4;
+  const unsigned long long pol = l2_prio<0, false>() >= 0 ? l2_policy(l2_prio<0, false>()) : 0ull;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ring, base, pa, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2, 0>(ring, base, pa, 16 * j, j, lane, pol);
     cp_async_commit();
   }
   const int fo = (lane >> 2) * SL + (lane & 3);  // fragment offset inside a column group
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2, 0>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane, pol);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
@@ -235,7 +279,7 @@ __device__ __forceinline__ void gram_tiles_async(double* ring, const double* bas
 
 // X <- X * J' for the global panel of pair (I, J), slabs streamed through the NS-stage ring; results
 // are stored straight to global memory (rows of a slab are read before they are overwritten).
-template <int W2, int NS>
+template <int W2, int NS, int K = 1>
 __device__ __forceinline__ void apply_rotation_async(double* ring, double* base, int ld, int rows, int I, int J,
                                                      int lane, const double (&jf)[W2 / 4][W2 / 8]) {
   constexpr int CG = W2 / 8, KK = W2 / 4, SL = WarpSmem<W2>::SL;
@@ -244,14 +288,16 @@ __device__ __forceinline__ void apply_rotation_async(double* ring, double* base,
   constexpr int W = W2 / 2, HB = CG / 2;
   const int oI = (I * W + 2 * (lane & 3)) * ld + (lane >> 2), oJ = (J * W + 2 * (lane & 3)) * ld + (lane >> 2);
   const int nslab = rows >> 4;
+  const unsigned long long pol = l2_prio<K, false>() >= 0 ? l2_policy(l2_prio<K, false>()) : 0ull;
+  const unsigned long long pst = l2_prio<K, true>() >= 0 ? l2_policy(l2_prio<K, true>()) : 0ull;
 #pragma unroll
   for (int j = 0; j < NS - 1; ++j) {
-    if (j < nslab) slab_issue<W2>(ring, base, pa, 16 * j, j, lane);
+    if (j < nslab) slab_issue<W2, K>(ring, base, pa, 16 * j, j, lane, pol);
     cp_async_commit();
   }
   const int fo = (lane & 3) * SL + (lane >> 2);  // A fragment: row l/4, column l%4
   for (int sl = 0; sl < nslab; ++sl) {
-    if (sl + NS - 1 < nslab) slab_issue<W2>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane);
+    if (sl + NS - 1 < nslab) slab_issue<W2, K>(ring, base, pa, 16 * (sl + NS - 1), (sl + NS - 1) % NS, lane, pol);
     cp_async_commit();
     cp_async_wait<NS - 1>();
     __syncwarp();
@@ -271,9 +317,11 @@ __device__ __forceinline__ void apply_rotation_async(double* ring, double* base,
 #pragma unroll
       for (int nb = 0; nb < CG; ++nb)
 #pragma unroll
-        for (int e = 0; e < 2; ++e)
-          __stcg(base + (nb < HB ? oI + (8 * nb + e) * ld : oJ + (8 * (nb - HB) + e) * ld) + 16 * sl + 8 * h,
-                 acc[nb][e]);
+        for (int e = 0; e < 2; ++e) {
+          double* dst = base + (nb < HB ? oI + (8 * nb + e) * ld : oJ + (8 * (nb - HB) + e) * ld) + 16 * sl + 8 * h;
+          if constexpr (l2_prio<K, true>() >= 0) st_hint(dst, acc[nb][e], pst);
+          else __stcg(dst, acc[nb][e]);
+        }
     }
     __syncwarp();
   }
@@ -746,6 +794,22 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(1);
   PHASE_COUNT(7);
   if (!__any_sync(0xffffffffu, need)) return false;
+#ifdef WCSVD_PHASE_PROFILE
+  {  // how close to diagonal is B? max over rotating pairs of |b_pq| / |b_pp - b_qq| (experiment)
+    double mx = 0.0;
+    if (lane < W2) {
+      const double bqq = B0[lane * W2 + lane];
+      for (int p = 0; p < lane; ++p) {
+        const double bpp = B0[p * W2 + p], bpq = B0[p * W2 + lane];
+        if (bpq * bpq > tol2 * bpp * bqq) mx = fmax(mx, fabs(bpq) / fabs(bpp - bqq));
+      }
+    }
+    for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if (mx <= 1e-2) PHASE_COUNT(10);
+    if (mx <= 2e-3) PHASE_COUNT(9);
+    if (mx <= 1e-4) PHASE_COUNT(11);
+  }
+#endif
   // (2) EVD of B (Alg 1 l.6): threshold parallel Jacobi, B and J in slot order.
   double ja[W2], jb[W2];
   bool rotated = false;
@@ -855,9 +919,9 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(3);
   // (3) A_ij <- A_ij J (Alg 1 l.7) and V_ij <- V_ij J.
   __syncwarp();  // the ring aliases B: every lane holds its J' fragments before slabs land
-  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE>(ws.ring, Wm, ld, mrows, I, J, lane, jf);
+  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE, 1>(ws.ring, Wm, ld, mrows, I, J, lane, jf);
   PHASE_MARK(4);
-  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE>(ws.ring, Vm, ldv, vrows, I, J, lane, jf);
+  apply_rotation_async<W2, WarpSmem<W2>::NSTAGE, 2>(ws.ring, Vm, ldv, vrows, I, J, lane, jf);
   PHASE_MARK(5);
   return true;
 }

@@ -19,3 +19,4 @@ for i, n in enumerate(names):
     print(f"{n:9s} {buf[i]/tot*100:5.1f}%  {buf[i]:.3e} warp-cycles")
 print(f"EVD steps {buf[6]*31}, rotation-free {buf[8]} ({100*buf[8]/max(buf[6]*31,1):.1f}%)")
 print(f"pairs {buf[7]}, with EVD {buf[6]}; cycles/pair {tot/max(buf[7],1):.0f}; EVD cycles/call {buf[2]/max(buf[6],1):.0f}; gram/pair {buf[0]/max(buf[7],1):.0f}; apply_A/call {buf[4]/max(buf[6],1):.0f} apply_V/call {buf[5]/max(buf[6],1):.0f}")
+print(f"near-diagonal B among pairs with an EVD: <=1e-2 {buf[10]/max(buf[6],1)*100:.1f}%  <=2e-3 {buf[9]/max(buf[6],1)*100:.1f}%  <=1e-4 {buf[11]/max(buf[6],1)*100:.1f}%")

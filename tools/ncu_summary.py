@@ -99,6 +99,10 @@ def main():
         except Exception:
             allj = {}
         s["dram_bytes_per_launch"] = (s["dram_read_bytes"] or 0) + (s["dram_write_bytes"] or 0)
+        if "--matrices" in sys.argv:  # matrices factored by the captured launch (grid / CTAs per matrix)
+            nm = int(sys.argv[sys.argv.index("--matrices") + 1])
+            s["matrices"] = nm
+            s["dram_bytes_per_matrix"] = s["dram_bytes_per_launch"] / nm
         s["report"] = rep
         allj[key] = s
         json.dump(allj, open(out, "w"), indent=1)
