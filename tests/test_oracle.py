@@ -181,6 +181,33 @@ def test_p11_transpose_symmetry_is_bitwise():
             assert np.abs(r.S - rt.S).max() <= 8 * U53 * r.S[0]
 
 
+def test_z15_sign_rule_fixes_the_square_factor():
+    # Z15 (oracle step 8): singular vectors are unique only up to a joint sign; the sign rule (largest-|.|
+    # entry of each square-factor column positive, first on ties) makes them a function of A alone. Pin:
+    # permuting the columns of a tall A (A P = U S (P^T V)^T) must return P^T V and the same U without
+    # any sign alignment, and permuting the rows of a wide A (P A = (P U) S V^T) must return P U and the
+    # same V -- the Jacobi iteration on the permuted matrix takes a different rotation sequence, so only
+    # the rule (applied to the right factor, on the right entry) can make the signs agree.
+    rng = np.random.default_rng(52)
+    for (m, n) in ((30, 12), (12, 30)):
+        A = workloads.prescribed(rng, m, n, np.geomspace(1.0, 1e-2, min(m, n)))  # well-separated sigma
+        r = oracle.svd(A)
+        if m >= n:
+            p = rng.permutation(n)
+            rp = oracle.svd(A[:, p].copy())
+            Vexp, Uexp = r.V[p, :], r.U
+            assert np.abs(rp.V - Vexp).max() <= 1e-12 and np.abs(rp.U - Uexp).max() <= 1e-12
+        else:
+            p = rng.permutation(m)
+            rp = oracle.svd(A[p, :].copy())
+            Uexp, Vexp = r.U[p, :], r.V
+            assert np.abs(rp.U - Uexp).max() <= 1e-12 and np.abs(rp.V - Vexp).max() <= 1e-12
+        assert np.abs(rp.S - r.S).max() <= 8 * U53 * r.S[0]
+        # and the rule itself: every square-factor column's largest-|.| entry (first on ties) is > 0
+        Q = rp.V if m >= n else rp.U
+        assert all(Q[np.argmax(np.abs(Q[:, j])), j] > 0 for j in range(Q.shape[1]))
+
+
 def test_z14_rank_deficient_completion():
     rng = np.random.default_rng(51)
     # exact zero columns, and an exactly rank-2 product
