@@ -222,135 +222,6 @@ __device__ __forceinline__ void x_sweep(TPCtx<T>& cx, T (&a)[R][NP / G], T (&b)[
   }
 }
 
-// ---- Warp-local X step (TPCfg WL = true) ----
-// Thread t holds rows 4 (t % 16) .. +3 of column group g = t / 16: a half-warp owns ALL rows of a
-// group, so gamma_k (and alpha, beta at a sweep's first step) are summed by a fixed shuffle tree
-// inside the half-warp (reduce-scatter over xor 8 / 4, then xor 2 / 1: every lane ends with the full
-// sum of local pair 2 b3 + b2, bitwise equal in the four lanes that hold it), the rotation is
-// evaluated in-warp (eq (4), R-ROT) and read back by the half-warp from the stored sweep record;
-// only the two ring elements that cross a warp boundary go through shared memory, behind one CTA
-// barrier per step (the fused reduction keeps no serial warp and no second barrier).
-template <typename T>
-__device__ __forceinline__ T shx(T v, int m) { return __shfl_xor_sync(0xffffffffu, v, m); }
-
-// reduce-scatter of v[0..3] over the 16 lanes of a half-warp: returns the total of v[2 b3 + b2]
-template <typename T>
-__device__ __forceinline__ T hw_reduce4(const T (&v)[4], int lane) {
-  const bool b3 = (lane >> 3) & 1, b2 = (lane >> 2) & 1;
-  const T k0 = (b3 ? v[2] : v[0]) + shx(b3 ? v[0] : v[2], 8);
-  const T k1 = (b3 ? v[3] : v[1]) + shx(b3 ? v[1] : v[3], 8);
-  const T m = (b2 ? k1 : k0) + shx(b2 ? k0 : k1, 4);
-  const T t = m + shx(m, 2);
-  return t + shx(t, 1);
-}
-
-template <typename T, int NP, int G, int R, bool FIRST>
-__device__ __forceinline__ void x_step_wl(TPCtx<T>& cx, const T (&x)[R][NP / G], T (&y)[R][NP / G], int step,
-                                          T* __restrict__ xo) {
-  constexpr int NL = NP / G;
-  constexpr int LP = NL / 2;
-  static_assert(LP == 4 && R == 4, "warp-local layout: 16 row-threads x 4 rows x 4 pairs per group");
-  using V2 = typename Prec<T>::V2;
-  const int g = cx.g, rt = cx.rt, lane = cx.lane;
-  TP_T(t0);
-  // (1) partial dot products over this thread's rows (all rows of the group live in the half-warp)
-  T gm[LP], al[LP], be[LP];
-#pragma unroll
-  for (int j = 0; j < LP; ++j) gm[j] = al[j] = be[j] = 0;
-#pragma unroll
-  for (int r = 0; r < R; ++r)
-#pragma unroll
-    for (int j = 0; j < LP; ++j) {
-      gm[j] = fma(x[r][2 * j], x[r][2 * j + 1], gm[j]);
-      if (FIRST) {
-        al[j] = fma(x[r][2 * j], x[r][2 * j], al[j]);
-        be[j] = fma(x[r][2 * j + 1], x[r][2 * j + 1], be[j]);
-      }
-    }
-  // (2) fixed-order half-warp reduction; this lane then owns local pair jj
-  const int jj = ((lane >> 3) & 1) * 2 + ((lane >> 2) & 1);
-  const int k = g * LP + jj;  // global pair = slots (2k, 2k+1)
-  const T gsum = hw_reduce4<T>(gm, lane);
-  T a, b;
-  if (FIRST) {
-    a = hw_reduce4<T>(al, lane);
-    b = hw_reduce4<T>(be, lane);
-  } else {
-    a = cx.nrm[cx.par * NP + 2 * k];
-    b = cx.nrm[cx.par * NP + 2 * k + 1];
-  }
-  T c, sn, t;
-  const bool rot = jacobi_rotation(a, b, gsum, cx.tol2, c, sn, t);
-  V2* rs = cx.rot + step * (G * (LP + 1)) + g * (LP + 1);
-  if ((lane & 3) == 0) {
-    rs[jj] = Prec<T>::mk(c, sn);
-    // eq (6) in closed form, written to the slots the two columns move to
-    cx.nrm[(cx.par ^ 1) * NP + rr_dest(2 * k, NP)] = rot ? fma(t, gsum, a) : a;
-    cx.nrm[(cx.par ^ 1) * NP + rr_dest(2 * k + 1, NP)] = rot ? fma(-t, gsum, b) : b;
-  }
-  if (__any_sync(0xffffffffu, rot) && lane == 0) *cx.rot_flag = 1;
-  __syncwarp();
-  TP_T(t1);
-  // (3) rotate this thread's rows (eq 3) and move along the ring (as rotate_move)
-  T top0[R], send_l[R], send_r[R];
-#pragma unroll
-  for (int j = 0; j < LP; ++j) {
-    const V2 p = rs[j];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      const T aa = x[r][2 * j], bb = x[r][2 * j + 1];
-      const T na = fma(p.y, bb, p.x * aa);
-      const T nb = fma(-p.y, aa, p.x * bb);
-      if (j == 0) top0[r] = na;
-      else if (j + 1 < LP) y[r][2 * (j + 1)] = na;
-      else send_r[r] = na;
-      if (j == 0) send_l[r] = nb;
-      else y[r][2 * (j - 1) + 1] = nb;
-    }
-  }
-  // neighbours: g^1 is the other half of this warp (shuffle); the far neighbour is in the next /
-  // previous warp (shared memory): even g sends send_l left, odd g sends send_r right.
-  const bool odd = g & 1;
-  const bool gfirst = (g == 0), glast = (g == G - 1);
-  T from_in[R];
-  T* xw = xo + cx.par * (G * 16 * R);
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    from_in[r] = shx(odd ? send_l[r] : send_r[r], 16);
-    xw[(g * 16 + rt) * R + r] = odd ? send_r[r] : send_l[r];
-  }
-  TP_T(t2);
-  __syncthreads();
-  const int src = odd ? g + 1 : g - 1;  // the group whose cross-warp value this thread receives
-  const bool has_src = odd ? !glast : !gfirst;
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    const T from_x = has_src ? xw[(src * 16 + rt) * R + r] : T(0);
-    const T from_left = odd ? from_in[r] : from_x;
-    const T from_right = odd ? from_x : from_in[r];
-    y[r][0] = gfirst ? top0[r] : from_left;
-    y[r][2] = gfirst ? send_l[r] : top0[r];
-    y[r][2 * (LP - 1) + 1] = glast ? send_r[r] : from_right;
-  }
-  cx.par ^= 1;
-#ifdef WCSVD_PHASE_PROFILE
-  TP_T(t3);
-  cx.acc[0] += t1 - t0;  // partials + reduction + rotation (reported as "phase1+bar1")
-  cx.acc[1] += t3 - t2;  // barrier + receive (reported as "serial+bar2")
-  cx.acc[2] += t2 - t1;  // rotate + hand-off (reported as "rotate")
-#endif
-}
-
-template <typename T, int NP, int G, int R>
-__device__ __forceinline__ void x_sweep_wl(TPCtx<T>& cx, T (&a)[R][NP / G], T (&b)[R][NP / G], T* xo) {
-  x_step_wl<T, NP, G, R, true>(cx, a, b, 0, xo);
-#pragma unroll 1
-  for (int s = 1; s < NP - 1; s += 2) {
-    x_step_wl<T, NP, G, R, false>(cx, b, a, s, xo);
-    x_step_wl<T, NP, G, R, false>(cx, a, b, s + 1, xo);
-  }
-}
-
 // V phase: replay the sweep's stored rotations on this thread's row of V (R = 1 row, NP/GV slots).
 // `rot` + the group offset of this thread; the stored layout is the X phase's [GX][LPX+1] per step.
 // PACKED: the rotations are stored as [NPAIR] per step, else as the X phase's padded [GX][LPX+1].
@@ -444,10 +315,9 @@ constexpr size_t l0tp_park_elems(int nt) {
 // One CTA per matrix. X phase: thread t = (row-thread rt = t / GX, group g = t % GX) holds rows
 // rt*RX .. rt*RX+RX-1 x slots g*NP/GX .. of X. V phase: thread t = (row rv = t / GV, group
 // gv = t % GV) holds row rv x slots gv*NP/GV .. of V_x.
-template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB, bool WL>
+template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB>
 __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restrict__ descs,
                                                           const int* __restrict__ order, SlotPool pool) {
-  static_assert(!WL || (!RED && RX == 4 && NP / GX == 8 && MAXT == 16 * GX), "warp-local layout");
   using V2 = typename Prec<T>::V2;
   constexpr int NLX = NP / GX;
   constexpr int LPX = NLX / 2;
@@ -461,8 +331,8 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
   const int NT = blockDim.x;
   const int tid = threadIdx.x;
   const int lane = tid & 31, warp = tid >> 5;
-  // X-phase layout: row-thread rt = t / GX, group g = t % GX; warp-local (WL): g = t / 16, rt = t % 16
-  const int g = WL ? tid / 16 : tid % GX, rt = WL ? tid % 16 : tid / GX;
+  // X-phase layout: row-thread rt = t / GX, group g = t % GX
+  const int g = tid % GX, rt = tid / GX;
   const bool isW = rt < RW;
   const int gv = tid % GV, rv = tid / GV;
   const bool withv = d.withv != 0;
@@ -555,8 +425,7 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
       // this sweep's flag was cleared one sweep earlier (or at start); clear the next one (its last
       // readers passed the barrier that ended the previous loop iteration)
       if (tid == 0) s_flags[4 + ((sweep + 1) & 1)] = 0;
-      if constexpr (WL) x_sweep_wl<T, NP, GX, RX>(cx, xa, xb, s_part);
-      else x_sweep<T, NP, GX, RX, RED, (MAXT / GX + 3) / 4 * 4>(cx, xa, xb);  // ends in xb, slots in order
+      x_sweep<T, NP, GX, RX, RED, (MAXT / GX + 3) / 4 * 4>(cx, xa, xb);  // ends in xb, slots in order
       ++sweep;
       __syncthreads();
       const bool any = *cx.rot_flag != 0;
@@ -606,10 +475,6 @@ __global__ void __launch_bounds__(MAXT, MINB) l0tp_kernel(const MatDesc* __restr
   // ---- Finalisation: sigma_j = ||x_j|| (fresh, fixed order), stable descending
   // rank (Z15), U = X / sigma, sign rule on the square factor V_x (Z15), un-orientation.
   __syncthreads();
-  if constexpr (WL) {  // the ring hand-off buffer aliased s_part: rows RW .. RW4-1 must read as zero
-    for (int e = tid; e < 3 * RW4 * PS; e += NT) s_part[e] = T(0);
-    __syncthreads();
-  }
   if (isW) {
 #pragma unroll
     for (int l = 0; l < NLX; ++l) {
@@ -730,13 +595,13 @@ constexpr int tp_threads(int M) {
   return (((M + RX - 1) / RX * GX > NP * GV ? (M + RX - 1) / RX * GX : NP * GV) + 31) / 32 * 32;
 }
 
-template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB, bool WL>
+template <typename T, int NP, int GX, int RX, int GV, bool RED, int MAXT, int MINB>
 static cudaError_t launch_tp_t(const MatDesc* descs, const int* order, int count, int maxM, const SlotPool& pool,
                                cudaStream_t stream) {
   const int threads = tp_threads<NP, GX, RX, GV>(maxM);
   if (threads > MAXT) return cudaErrorInvalidConfiguration;
   const size_t smem = l0tp_smem_bytes<T, NP, GX, RX, RED>(maxM, threads);
-  auto kern = l0tp_kernel<T, NP, GX, RX, GV, RED, MAXT, MINB, WL>;
+  auto kern = l0tp_kernel<T, NP, GX, RX, GV, RED, MAXT, MINB>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   kern<<<count, threads, smem, stream>>>(descs, order, pool);
@@ -746,33 +611,23 @@ static cudaError_t launch_tp_t(const MatDesc* descs, const int* order, int count
 // Variant configurations: X layout (GX groups, RX rows per thread), V layout (GV groups, one row
 // per thread), rotation evaluation (RED: every warp, else one warp), launch bounds. The planner's M
 // limits (kernels.h) bound the thread count of every bucket.
-#ifndef WCSVD_TP64_CFG
-#define WCSVD_TP64_CFG 0
-#endif
+// Variant configurations: X layout (GX groups, RX rows per thread), V layout (GV groups, one row
+// per thread), rotation evaluation (RED: every warp, else one warp), launch bounds. Measured
+// alternatives for NP = 64 (r01): every warp reduces (RED, 128 threads) 24.4 ms,
+// 8 rows per thread with 64 threads 21.6 ms, warp-local X step (a half-warp owns all rows of a group,
+// shuffle-tree reduction) 19.5 ms, against 18.8 ms for the layout below.
 template <int V>
 struct TPCfg;
 template <>
 struct TPCfg<kTP32> {  // 32-column matrices: one warp holds a 32 x 32 X (R = 4)
   static constexpr int NP = 32, GX = 4, RX = 4, GV = 1, MAXT = 128, MINB = 4;
-  static constexpr bool RED = true, WL = false;
+  static constexpr bool RED = true;
   static constexpr int kMaxM = kTP32MaxM;
 };
 template <>
-struct TPCfg<kTP64> {
-#if WCSVD_TP64_CFG == 0
+struct TPCfg<kTP64> {  // 64-column matrices: 8 column groups x 16 row-threads x 4 rows; V: 2 groups x 64 rows
   static constexpr int NP = 64, GX = 8, RX = 4, GV = 2, MAXT = 128, MINB = 4;
-  static constexpr bool RED = false, WL = false;
-#elif WCSVD_TP64_CFG == 2
-  static constexpr int NP = 64, GX = 8, RX = 4, GV = 2, MAXT = 128, MINB = 4;
-  static constexpr bool RED = true, WL = false;
-#elif WCSVD_TP64_CFG == 3
-  // warp-local X step: a half-warp owns all 64 rows of an 8-column group
-  static constexpr int NP = 64, GX = 8, RX = 4, GV = 2, MAXT = 128, MINB = 4;
-  static constexpr bool RED = false, WL = true;
-#else
-  static constexpr int NP = 64, GX = 8, RX = 8, GV = 1, MAXT = 64, MINB = 4;
-  static constexpr bool RED = true, WL = false;
-#endif
+  static constexpr bool RED = false;
   static constexpr int kMaxM = kTP64MaxM;
 };
 
@@ -798,7 +653,7 @@ static int occupancy_v(int maxM) {
   using C = TPCfg<V>;
   const int threads = tp_threads<C::NP, C::GX, C::RX, C::GV>(maxM);
   const size_t smem = l0tp_smem_bytes<T, C::NP, C::GX, C::RX, C::RED>(maxM, threads);
-  auto kern = l0tp_kernel<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB, C::WL>;
+  auto kern = l0tp_kernel<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB>;
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) return -1;
   int nb = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads, smem) != cudaSuccess) return -1;
@@ -818,8 +673,7 @@ template <typename T, int V>
 static cudaError_t launch_v(const MatDesc* descs, const int* order, int count, int maxM, const SlotPool& pool,
                             cudaStream_t stream) {
   using C = TPCfg<V>;
-  return launch_tp_t<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB, C::WL>(descs, order, count, maxM, pool,
-                                                                                    stream);
+  return launch_tp_t<T, C::NP, C::GX, C::RX, C::GV, C::RED, C::MAXT, C::MINB>(descs, order, count, maxM, pool, stream);
 }
 
 cudaError_t launch_l0tp(int variant, int fp32, const MatDesc* descs, const int* order, int count, int maxM,
