@@ -88,7 +88,11 @@ struct PairCfg {
   static constexpr int W = W2 / 2;          // block width w
   static constexpr int CG = W2 / 8;         // 8-column groups per pair panel
   static constexpr int NTU = CG * (CG + 1) / 2;  // upper tiles of the 2w x 2w Gram
-  static constexpr int BS = W2 + 1;         // SMEM row stride of 2w x 2w buffers (doubles)
+  // SMEM row stride of the 2w x 2w J / E / J' buffers (doubles). W2 + 3: the Newton-Schulz fragment
+  // loads ((8i + l/4) BS + 4kk + l%4 and (4kk + l%4) BS + 8j + l/4), the J' stores and the J staging
+  // stores take 3 / 3 / 3 / 2 wavefronts per warp access instead of 4 / 4 / 4 / 2 with W2 + 1 (bank
+  // model in DESIGN.md §5.2); the EVD's full-symmetric B uses its own stride W2.
+  static constexpr int BS = W2 + 3;
   static_assert(W2 == 16 || W2 == 32, "pair panel width");
 };
 
