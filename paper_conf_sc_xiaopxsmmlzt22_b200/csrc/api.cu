@@ -24,6 +24,10 @@ namespace {
 constexpr int kMaxDim = 1024;
 constexpr int kHostSets = 4;         // max device staging sets of the host-buffer pipeline
 constexpr int kHostSetsDefault = 3;
+// host API: zero-copy route above this estimated flop / byte of I/O (10 sweeps x F_tb over A + S + U + V
+// bytes). Measured e2e (B200, matrices/s, staged pipeline vs zero-copy): C5 (1648 flop/B) 956 vs 1032;
+// C3 (743) 8983 vs 8022; C4 (327) 11481 vs 9543; C2 (183) 487k vs 144k.
+constexpr double kZeroCopyFlopPerByte = 1200.0;
 
 double f_tb(int M, int N) { return 0.5 * N * (N - 1.0) * (8.0 * M + 6.0 * N); }
 
@@ -609,6 +613,82 @@ cudaError_t copy_run(const HostRun& r, bool h2d, double* dev, const std::vector<
 
 }  // namespace
 
+// Device-visible alias of a host pointer if it is page-locked and mapped (cudaHostAlloc / torch
+// pin_memory under UVA), else nullptr (pageable memory: the staged pipeline is used).
+static void* mapped_alias(const void* p) {
+  if (!p) return nullptr;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return (at.type == cudaMemoryTypeHost && at.devicePointer) ? at.devicePointer : nullptr;
+}
+
+// Zero-copy route of wcsvd_batched_host: every host buffer is mapped, so the kernels
+// read A and write S, U, V in host memory themselves -- the host <-> device transfers happen inside
+// the kernels (stage-in reads A once, finalisation writes each output once) and overlap the other
+// CTAs' sweeps, with no staging copies and no chunk boundaries. Returns 1 if the route does not apply.
+static int batched_host_zero_copy(int batch, const int* m, const int* n, const double* const* A, const int* lda,
+                                  double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
+                                  cudaStream_t stream, const wcsvd_opts* opts) {
+  // policy: compute-heavy batches only (estimated flops per byte of I/O; the Level-0-sized ones keep
+  // the copy-engine pipeline, whose transfers already hide behind their short kernels). Env
+  // WCSVD_HOST_ZEROCOPY=0/1 forces the choice (experiments).
+  const char* env = std::getenv("WCSVD_HOST_ZEROCOPY");
+  if (env && std::atoi(env) == 0) return 1;
+  double fl = 0, by = 0;
+  for (int b = 0; b < batch; ++b) {
+    const int M = std::max(m[b], n[b]), N = std::min(m[b], n[b]);
+    fl += 10.0 * f_tb(M, N);
+    by += 8.0 * ((double)m[b] * n[b] + (double)N * (m[b] + n[b] + 1));
+  }
+  if (!(env && std::atoi(env) == 1) && fl < kZeroCopyFlopPerByte * by) return 1;
+  std::vector<const double*> pA(batch);
+  std::vector<double*> pS(batch), pU(U ? batch : 0), pV(V ? batch : 0);
+  for (int b = 0; b < batch; ++b) {
+    pA[b] = static_cast<const double*>(mapped_alias(A[b]));
+    pS[b] = static_cast<double*>(mapped_alias(S[b]));
+    if (!pA[b] || !pS[b]) return 1;
+    if (U && !(pU[b] = static_cast<double*>(mapped_alias(U[b])))) return 1;
+    if (V && !(pV[b] = static_cast<double*>(mapped_alias(V[b])))) return 1;
+  }
+  int* h_info = opts ? opts->info : nullptr;  // HOST int[batch] (may be pageable)
+  int* d_info = nullptr;
+  if (h_info && lib_malloc(reinterpret_cast<void**>(&d_info), sizeof(int) * (size_t)batch, stream) != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ENOMEM;
+  }
+  wcsvd_opts o;
+  std::memset(&o, 0, sizeof(o));
+  o.struct_size = sizeof(o);
+  o.info = d_info;
+  if (opts) {
+    o.ldu = opts->ldu;
+    o.ldv = opts->ldv;
+    o.force_path = opts->force_path;
+    o.force_w = opts->force_w;
+    o.wcycle_sweeps = opts->wcycle_sweeps;
+    o.inner_sweeps = opts->inner_sweeps;
+    o.pair_warps = opts->pair_warps;
+    o.cluster_ctas = opts->cluster_ctas;
+    o.f32_compute = opts->f32_compute;
+  }
+  const int rc = batched_impl<double>(batch, m, n, pA.data(), lda, pS.data(), U ? pU.data() : nullptr,
+                                      V ? pV.data() : nullptr, tol, max_sweeps,
+                                      reinterpret_cast<wcsvd_stream_t>(stream), &o);
+  cudaError_t e = cudaSuccess;
+  if (rc == WCSVD_OK && h_info) e = cudaMemcpyAsync(h_info, d_info, sizeof(int) * (size_t)batch, cudaMemcpyDeviceToHost, stream);
+  if (d_info) cudaFreeAsync(d_info, stream);
+  const cudaError_t es2 = cudaStreamSynchronize(stream);  // synchronous API: outputs are in host memory
+  if (rc != WCSVD_OK) return rc;
+  if (e != cudaSuccess || es2 != cudaSuccess) {
+    cudaGetLastError();
+    return WCSVD_ECUDA;
+  }
+  return WCSVD_OK;
+}
+
 static int batched_host_impl(int batch, const int* m, const int* n, const double* const* A, const int* lda,
                              double* const* S, double* const* U, double* const* V, double tol, int max_sweeps,
                              wcsvd_stream_t stream_, const wcsvd_opts* opts) {
@@ -621,6 +701,10 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   const bool wantU = U != nullptr, wantV = V != nullptr;
   for (int b = 0; b < batch && (wantU || wantV); ++b)
     if ((wantU && !U[b]) || (wantV && !V[b])) return -7;  // host API: a factor is requested for all or none
+  {
+    const int zc = batched_host_zero_copy(batch, m, n, A, lda, S, U, V, tol, max_sweeps, stream, opts);
+    if (zc != 1) return zc;
+  }
 
   // device staging offsets (packed per matrix, in batch order)
   std::vector<size_t> oA(batch), oS(batch), oU(batch), oV(batch);

@@ -55,6 +55,28 @@ def test_host_mixed_chunked_bitwise_equals_device():
     assert np.array_equal(info, infod.cpu().numpy()) and (info > 0).all()
 
 
+@pytest.mark.parametrize("route", ["1", "0"])
+def test_host_zero_copy_and_staged_routes_bitwise_equal_device(route, monkeypatch):
+    # the zero-copy route (every host buffer mapped: kernels read A / write S, U, V in host memory) and
+    # the staged pipeline must both return the device entry point's bits; pageable outputs make the
+    # zero-copy route fall back to the pipeline
+    monkeypatch.setenv("WCSVD_HOST_ZEROCOPY", route)
+    shapes = [(130, 100), (100, 150), (256, 256), (64, 64), (300, 170), (40, 24), (1024, 96), (97, 301)]
+    mats = [torch.from_numpy(workloads.gaussian(workloads.matrix_rng(910, k), m, n)).pin_memory()
+            for k, (m, n) in enumerate(shapes)]
+    Sd, Ud, Vd, infod = wc.svd_batched([a.cuda() for a in mats], return_info=True)
+    torch.cuda.synchronize()
+    for pinned_out in (True, False):
+        ks = [min(m, n) for (m, n) in shapes]
+        out = ([torch.empty(k, dtype=torch.float64, pin_memory=pinned_out) for k in ks],
+               [torch.empty(k, m, dtype=torch.float64, pin_memory=pinned_out) for k, (m, _) in zip(ks, shapes)],
+               [torch.empty(k, n, dtype=torch.float64, pin_memory=pinned_out) for k, (_, n) in zip(ks, shapes)])
+        S, U, V, info = wc.svd_batched_host(mats, return_info=True, out=out)
+        for k in range(len(mats)):
+            assert torch.equal(S[k], Sd[k].cpu()) and torch.equal(U[k], Ud[k].cpu()) and torch.equal(V[k], Vd[k].cpu()), k
+        assert np.array_equal(info, infod.cpu().numpy()) and (info > 0).all()
+
+
 def test_host_values_only_and_preallocated_out():
     mats = workloads.get_config("C3", batch=20).matrices()
     A = torch.from_numpy(np.stack(mats)).pin_memory()
