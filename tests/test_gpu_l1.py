@@ -74,6 +74,16 @@ def test_l1_1024_rows_against_the_oracle():
     check_parity(mats, S, U, V, info)
 
 
+def test_l1_1024_square_against_the_oracle():
+    # the largest size of the boundary against the long-double oracle itself (~2 min of oracle time
+    # on one host core; tools/oracle_check_large.py runs three such matrices)
+    cfg = workloads.get_config("C5", batch=1)
+    mats = [cfg.make(0)]
+    assert mats[0].shape == (1024, 1024)
+    S, U, V, info = gpu_svd_list(mats)
+    check_parity(mats, S, U, V, info)
+
+
 def test_l1_bitwise_deterministic_across_batch_composition():
     mats = [workloads.gaussian(workloads.matrix_rng(540, i), 160, 140) for i in range(6)]
     S1, U1, V1, _ = gpu_svd_list(mats)
