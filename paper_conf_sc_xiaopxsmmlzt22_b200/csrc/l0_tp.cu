@@ -125,30 +125,59 @@ __device__ __forceinline__ void x_step(TPCtx<T>& cx, const T (&x)[R][NP / G], T 
   const int SEC = cx.RW4 * cx.PS;
   T* part = cx.part + (RED ? cx.par * 3 * SEC : 0);
   TP_T(t0);
-  if (cx.isW) {
+  {
     // rows outer, pairs inner: LP independent accumulation chains interleave (each still sums its
-    // rows in order 0 .. R-1)
-    const int base = cx.rt * cx.PS + cx.g * LP;
+    // rows in order 0 .. R-1); rows >= M (row-threads past RW) contribute zeros
     T gm[LP], al[LP], be[LP];
 #pragma unroll
     for (int j = 0; j < LP; ++j) gm[j] = al[j] = be[j] = 0;
+    if (cx.isW) {
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
+      for (int r = 0; r < R; ++r) {
 #pragma unroll
-      for (int j = 0; j < LP; ++j) {
-        gm[j] = fma(x[r][2 * j], x[r][2 * j + 1], gm[j]);
-        if (FIRST) {
-          al[j] = fma(x[r][2 * j], x[r][2 * j], al[j]);
-          be[j] = fma(x[r][2 * j + 1], x[r][2 * j + 1], be[j]);
+        for (int j = 0; j < LP; ++j) {
+          gm[j] = fma(x[r][2 * j], x[r][2 * j + 1], gm[j]);
+          if (FIRST) {
+            al[j] = fma(x[r][2 * j], x[r][2 * j], al[j]);
+            be[j] = fma(x[r][2 * j + 1], x[r][2 * j + 1], be[j]);
+          }
         }
       }
     }
+    if constexpr (!RED) {
+      // one-warp rotation evaluation: the 32 / G row-threads of a warp pre-sum their partials by a
+      // fixed xor tree (the same bits in every lane of a group), so the serial warp adds one partial
+      // per warp instead of one per row-thread
 #pragma unroll
-    for (int j = 0; j < LP; ++j) {
-      part[base + j] = gm[j];
-      if (FIRST) {
-        part[SEC + base + j] = al[j];
-        part[2 * SEC + base + j] = be[j];
+      for (int o = G; o < 32; o <<= 1)
+#pragma unroll
+        for (int j = 0; j < LP; ++j) {
+          gm[j] += __shfl_xor_sync(0xffffffffu, gm[j], o);
+          if (FIRST) {
+            al[j] += __shfl_xor_sync(0xffffffffu, al[j], o);
+            be[j] += __shfl_xor_sync(0xffffffffu, be[j], o);
+          }
+        }
+      if (cx.lane < G) {
+        const int base = cx.warp * cx.PS + cx.g * LP;
+#pragma unroll
+        for (int j = 0; j < LP; ++j) {
+          part[base + j] = gm[j];
+          if (FIRST) {
+            part[SEC + base + j] = al[j];
+            part[2 * SEC + base + j] = be[j];
+          }
+        }
+      }
+    } else if (cx.isW) {
+      const int base = cx.rt * cx.PS + cx.g * LP;
+#pragma unroll
+      for (int j = 0; j < LP; ++j) {
+        part[base + j] = gm[j];
+        if (FIRST) {
+          part[SEC + base + j] = al[j];
+          part[2 * SEC + base + j] = be[j];
+        }
       }
     }
   }
@@ -167,7 +196,7 @@ __device__ __forceinline__ void x_step(TPCtx<T>& cx, const T (&x)[R][NP / G], T 
       // RWM (compile time) >= RW4: fully unrolled, so the loads of a block issue back to back
 #pragma unroll
       for (int i = 0; i < RWM; i += 4) {  // rows [RW, RW4) are zero
-        if (i >= cx.RW4) break;
+        if (i >= (RED ? cx.RW4 : cx.nwarp)) break;  // !RED: one pre-summed partial per warp
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           g4[u] += part[(i + u) * PS + k];
