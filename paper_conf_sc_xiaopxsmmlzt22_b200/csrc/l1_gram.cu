@@ -39,6 +39,13 @@
 #ifndef WCSVD_EVD_FULL
 #define WCSVD_EVD_FULL 1
 #endif
+// Nearly diagonal pair Grams (R-PERT): when every rotating b_pq is below kPertDelta times
+// |b_pp - b_qq|, J is the first-order eigenvector matrix I + E (E_pq = b_pq / (b_qq - b_pp)) made
+// orthogonal by two Newton-Schulz steps, instead of the 2w-1-step Jacobi sweep. 0 disables it.
+#ifndef WCSVD_L1_PERT
+#define WCSVD_L1_PERT 1
+#endif
+constexpr double kPertDelta = 1e-4;
 // Inner EVD angle: 0 = exact fp64 eq (4) (R-ROT), 1 = fp32 angle with fp64-orthogonal (c, s) (R-ROT32)
 #ifndef WCSVD_EVD_ROT32
 #define WCSVD_EVD_ROT32 0
@@ -779,6 +786,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   PHASE_MARK(0);
   // (4) off-norm test on the Gram (Z6): skip the pair if every b_pq^2 <= tol^2 b_pp b_qq.
   bool need = false;
+  bool pert_ok = true;  // R-PERT: every rotating b_pq is small against its diagonal gap
   {
 #if WCSVD_EVD_FULL
 #define BIDX(a, b) ((a) * W2 + (b))
@@ -792,7 +800,9 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
       const double bpq = (lane < W2 && lane > p) ? B0[BIDX(p, lane)] : 0.0;
 #undef BIDX
       const double ab = bpp * bqq;
-      need |= (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
+      const bool rot = (lane > p && ab > 0.0 && bpq * bpq > tol2 * ab);
+      need |= rot;
+      pert_ok &= !rot || fabs(bpq) <= kPertDelta * fabs(bpp - bqq);
     }
   }
   PHASE_MARK(1);
@@ -819,6 +829,23 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   bool rotated = false;
   int isw = 0;
   bool panel_done = false;
+  const bool pert = WCSVD_L1_PERT && WCSVD_EVD_FULL && !PANEL && __all_sync(0xffffffffu, pert_ok);
+  if (pert) {
+    // R-PERT: lane p builds row p of J = I + E, E_pq = b_pq / (b_qq - b_pp) for the rotating pairs
+    // (the first-order eigenvectors of a nearly diagonal B; antisymmetric)
+    const double bpp = (lane < W2) ? B0[lane * W2 + lane] : 1.0;
+#pragma unroll
+    for (int q = 0; q < W2; ++q) {
+      const double bqq = B0[q * W2 + q];  // broadcast
+      const double bpq = (lane < W2) ? B0[lane * W2 + q] : 0.0;
+      const double ab = bpp * bqq;
+      const bool rot = q != lane && ab > 0.0 && bpq * bpq > tol2 * ab;
+      ja[q] = (q == lane) ? 1.0 : (rot ? bpq / (bqq - bpp) : 0.0);
+    }
+    rotated = true;
+    isw = 1;
+    panel_done = true;
+  }
   if constexpr (PANEL && W2 == 32) {
     // group (i): one-sided Jacobi of the (CholeskyQR-compressed) panel; group (ii) below if a pivot is tiny
     if (inner_cap == 1) panel_done = evd_fast32(B0, B1, lane, tol2, ja, &rotated);
@@ -868,7 +895,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
     if (!any) break;
   }
   }
-  *inner += isw + (isw < inner_cap ? 1 : 0);
+  *inner += pert ? 1 : isw + (isw < inner_cap ? 1 : 0);
   PHASE_MARK(2);
   PHASE_COUNT(6);
   if (!rotated) return false;
@@ -879,6 +906,14 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   }
   __syncwarp();
 #if WCSVD_L1_NS
+  for (int nsp = 0; nsp < (pert ? 2 : 1); ++nsp) {
+  if (nsp) {  // R-PERT: a second Newton-Schulz step on J' (J = I + E is orthogonal only to O(E^2))
+    if (lane < W2) {
+#pragma unroll
+      for (int s = 0; s < W2; ++s) ws.S[lane * BS + s] = ws.B[lane * BS + s];
+    }
+    __syncwarp();
+  }
   {
     const double* ptr[CG];
 #pragma unroll
@@ -911,6 +946,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
 #pragma unroll
       for (int e = 0; e < 2; ++e) ws.B[(8 * i + (lane >> 2)) * BS + 8 * j + 2 * (lane & 3) + e] = jn[i][j][e];
   __syncwarp();
+  }
   const double* jsrc = ws.B;
 #else
   const double* jsrc = ws.S;  // ablation build (-DWCSVD_L1_NS=0): J applied without the cleanup step
