@@ -45,7 +45,14 @@
 #ifndef WCSVD_L1_PERT
 #define WCSVD_L1_PERT 1
 #endif
-constexpr double kPertDelta = 1e-4;
+// (delta = 1e-3 with three Newton-Schulz steps covers more pairs but measured slower: C3 211.4 vs 208.6
+// ms, 12.39 vs 12.37 sweeps; half C5 1417 vs 1413 ms)
+#ifndef WCSVD_L1_PERT_DELTA
+#define WCSVD_L1_PERT_DELTA 1e-4
+#endif
+constexpr double kPertDelta = WCSVD_L1_PERT_DELTA;
+// Newton-Schulz steps after J = I + E: ||J^T J - I|| <= (2w delta)^2 shrinks as e -> 0.75 e^2 per step
+constexpr int kPertNS = kPertDelta <= 1e-4 ? 2 : 3;
 // Inner EVD angle: 0 = exact fp64 eq (4) (R-ROT), 1 = fp32 angle with fp64-orthogonal (c, s) (R-ROT32)
 #ifndef WCSVD_EVD_ROT32
 #define WCSVD_EVD_ROT32 0
@@ -906,7 +913,7 @@ __device__ bool process_pair(const WarpSmem<W2>& ws, const EvdMap<W2>* s_em, dou
   }
   __syncwarp();
 #if WCSVD_L1_NS
-  for (int nsp = 0; nsp < (pert ? 2 : 1); ++nsp) {
+  for (int nsp = 0; nsp < (pert ? kPertNS : 1); ++nsp) {
   if (nsp) {  // R-PERT: a second Newton-Schulz step on J' (J = I + E is orthogonal only to O(E^2))
     if (lane < W2) {
 #pragma unroll
