@@ -425,7 +425,7 @@ def main():
             "sweep_normalised_tflops": flops_all / (ms_step * 1e-3) / 1e12,
             "e2e": {"value": e2e_value, "unit": "matrices/s", "h2d_bytes_per_step": int(h2d_all),
                     "d2h_bytes_per_step": int(d2h_all),
-                    "what": "wcsvd_batched_host on every rank (pinned host A -> H2D -> kernels -> D2H of S, U, V)"
+                    "what": "wcsvd_batched_host on every rank (pinned host A in, S, U, V out: staged H2D / kernels / D2H pipeline, or for compute-heavy batches such as C5 the zero-copy route where the kernels read A and write S, U, V in the mapped host buffers; DESIGN.md 5.6)"
                             + (" + one NCCL all_gather of S to rank 0 (dist.gather_sigma)" if world > 1 else "")},
             "gpu_launches": int(launches) * args.steps,
             "clocks": clk.summary(),
