@@ -148,7 +148,8 @@ WCSVD_API int wcsvd_batched_f32_ex(int batch, const int* m, const int* n, const 
  * least 1), a mixed-size batch into 3 chunks when it has >= 300 matrices (else 1). Chunk c is copied in
  * (stream 1), factored on one of two compute streams, and copied out (stream 2) while later chunks are
  * copied in / factored, through three device staging sets (chunk c's H2D waits for the D2H of chunk
- * c-3). Host blocks of consecutive matrices that are adjacent and packed (ld = rows) move as one copy
+ * c-3); a batch of one chunk is copied in, factored and copied out in order on `stream` (no pipeline
+ * streams to set up). Host blocks of consecutive matrices that are adjacent and packed (ld = rows) move as one copy
  * (per matrix if the runtime refuses a merged range).
  * Zero-copy route: when EVERY host buffer is page-locked and mapped into the device address space
  * (cudaHostAlloc / cudaMallocHost / torch pin_memory under UVA) and the batch is compute-heavy (estimated

@@ -772,12 +772,86 @@ static int batched_host_impl(int batch, const int* m, const int* n, const double
   int NSET = kHostSetsDefault;
   if (const char* env = std::getenv("WCSVD_HOST_SETS")) NSET = std::max(2, std::min(kHostSets, std::atoi(env)));  // experiments
   NSET = std::min(NSET, std::max(2, C));
+  int* h_info = opts ? opts->info : nullptr;  // HOST int[batch] for this entry point
+  if (C == 1) {
+    // One chunk (small batches, e.g. C1): copy in, factor and copy out in order on the caller's stream
+    // -- no pipeline streams or events to create (their setup cost ~0.3 ms per call, as much as C1's
+    // kernels), one staging set.
+    double* d1 = nullptr;
+    if (lib_malloc(reinterpret_cast<void**>(&d1), setB, stream) != cudaSuccess) {
+      cudaGetLastError();
+      return WCSVD_ENOMEM;
+    }
+    double* dA = d1;
+    double* dS = dA + mxA;
+    double* dU = dS + mxS;
+    double* dV = dU + mxU;
+    int* dI = reinterpret_cast<int*>(dV + mxV);
+    cudaError_t x = cudaSuccess;
+    for (const HostRun& r : host_runs(0, batch, oA, A, m, n, lda, mergeA)) {
+      if (x != cudaSuccess) break;
+      x = copy_run(r, true, dA, oA, A, m, n, lda, stream);
+    }
+    int rc1 = WCSVD_OK;
+    if (x == cudaSuccess) {
+      std::vector<const double*> pA(batch);
+      std::vector<double*> pS(batch), pU(wantU ? batch : 0), pV(wantV ? batch : 0);
+      std::vector<int> ld_(batch);
+      for (int b = 0; b < batch; ++b) {
+        pA[b] = dA + oA[b];
+        ld_[b] = m[b];
+        pS[b] = dS + oS[b];
+        if (wantU) pU[b] = dU + oU[b];
+        if (wantV) pV[b] = dV + oV[b];
+      }
+      wcsvd_opts o;
+      std::memset(&o, 0, sizeof(o));
+      o.struct_size = sizeof(o);
+      o.info = h_info ? dI : nullptr;
+      if (opts) {
+        o.force_path = opts->force_path;
+        o.force_w = opts->force_w;
+        o.wcycle_sweeps = opts->wcycle_sweeps;
+        o.inner_sweeps = opts->inner_sweeps;
+        o.pair_warps = opts->pair_warps;
+        o.cluster_ctas = opts->cluster_ctas;
+        o.f32_compute = opts->f32_compute;
+      }
+      rc1 = batched_impl<double>(batch, m, n, pA.data(), ld_.data(), pS.data(), wantU ? pU.data() : nullptr,
+                                 wantV ? pV.data() : nullptr, tol, max_sweeps, stream_, &o, tot);
+    }
+    if (x == cudaSuccess && rc1 == WCSVD_OK) {
+      for (const HostRun& r : host_runs(0, batch, oS, S, kk.data(), ones.data(), kk.data(), mergeS)) {
+        if (x != cudaSuccess) break;
+        x = copy_run(r, false, dS, oS, S, kk.data(), ones.data(), kk.data(), stream);
+      }
+      if (wantU)
+        for (const HostRun& r : host_runs(0, batch, oU, U, m, kk.data(), ldu_v.data(), mergeU)) {
+          if (x != cudaSuccess) break;
+          x = copy_run(r, false, dU, oU, U, m, kk.data(), ldu_v.data(), stream);
+        }
+      if (wantV)
+        for (const HostRun& r : host_runs(0, batch, oV, V, n, kk.data(), ldv_v.data(), mergeV)) {
+          if (x != cudaSuccess) break;
+          x = copy_run(r, false, dV, oV, V, n, kk.data(), ldv_v.data(), stream);
+        }
+      if (h_info && x == cudaSuccess)
+        x = cudaMemcpyAsync(h_info, dI, sizeof(int) * (size_t)batch, cudaMemcpyDeviceToHost, stream);
+    }
+    cudaFreeAsync(d1, stream);
+    const cudaError_t es1 = cudaStreamSynchronize(stream);
+    if (rc1 != WCSVD_OK) return rc1;
+    if (x != cudaSuccess || es1 != cudaSuccess) {
+      cudaGetLastError();
+      return WCSVD_ECUDA;
+    }
+    return WCSVD_OK;
+  }
   double* dbuf = nullptr;
   if (lib_malloc(reinterpret_cast<void**>(&dbuf), NSET * setB, stream) != cudaSuccess) {
     cudaGetLastError();
     return WCSVD_ENOMEM;
   }
-  int* h_info = opts ? opts->info : nullptr;  // HOST int[batch] for this entry point
   cudaStream_t s_in = nullptr, s_out = nullptr, s_cp[2] = {nullptr, nullptr};
   cudaEvent_t ev_start = nullptr, ev_in[kHostSets] = {}, ev_cp[kHostSets] = {}, ev_out[kHostSets] = {};
   cudaError_t e = cudaStreamCreateWithFlags(&s_in, cudaStreamNonBlocking);
