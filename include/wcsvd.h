@@ -31,7 +31,9 @@
  *    max_sweeps) -- never on batch composition, stream, device index or device count. The plan is
  *    a function of (m, n) only; there are no floating-point atomics.
  *  - Reentrant. Process-wide state: only the per-device workspace pool above (created once, guarded
- *    by a mutex); nothing a call does changes another call's results.
+ *    by a mutex), the planner's immutable table coordinates, and, per host thread and device, the
+ *    streams / events of wcsvd_batched_host's pipeline (created on first use, drained by every call,
+ *    never shared between threads); nothing a call does changes another call's results.
  */
 #ifndef WCSVD_H_
 #define WCSVD_H_
